@@ -1,0 +1,64 @@
+// kernels.h - host-side launchers of the libmsort CUDA kernels (internal).
+#pragma once
+
+#include <cstddef>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace msort {
+
+inline int key_bytes(int kt) { return (kt == 1 || kt == 3) ? 8 : 4; }
+inline bool key_is_float(int kt) { return kt == 2 || kt == 3; }
+inline int num_passes(int kt) { return key_bytes(kt) * 8 / 8; }
+
+// ----- radix (S1-S3) ------------------------------------------------------
+struct RadixWs {
+    uint32_t* counters;           // [8] per-pass tile counters
+    uint32_t* hist;               // [8][256]
+    uint32_t* base;               // [8][256] exclusive digit bases
+    uint32_t* trivial;            // [8] 1 if the pass's digit is constant over all keys
+    unsigned long long* status;   // [tiles][256] decoupled-lookback words
+    uint64_t tiles;
+    size_t head_bytes;            // bytes of counters..trivial (zeroed per sort)
+};
+uint32_t radix_tile_keys(int kt);
+size_t radix_ws_bytes(uint64_t n, int kt);
+RadixWs radix_ws_layout(void* ws, uint64_t n, int kt);
+
+// Zero counters/hist/status, histogram all passes of `keys`, scan to bases,
+// set trivial flags.  keys are raw (T applied on load).
+cudaError_t radix_prologue(const void* keys, uint64_t n, int kt, const RadixWs& ws, cudaStream_t st);
+// histogram only into an external [P][256] array (zeroed inside)
+cudaError_t launch_histogram(const void* keys, uint64_t n, int kt, uint32_t* hist, cudaStream_t st);
+// bases from hist rows (all P)
+cudaError_t launch_scan(const uint32_t* hist, uint32_t* base, uint32_t* trivial, uint64_t n, int kt, cudaStream_t st);
+// one onesweep pass; flags: 1 = encode on load, 2 = decode on store
+cudaError_t launch_onesweep(const void* in, void* out, uint64_t n, int kt, int pass, int flags, const RadixWs& ws,
+                            const uint32_t* base_row, cudaStream_t st);
+
+// ----- merge phase (S4-S6) -------------------------------------------------
+struct GroupPtrs {
+    const void* p[8];
+};
+// Alg.1 for n_groups groups of `label` chunks each (group j = chunks [j*label, (j+1)*label)
+// of `all`); d_p[j] = pivot of group j.
+cudaError_t launch_pivots(const GroupPtrs& all, int n_groups, int label, uint64_t c, int kt, uint64_t* d_p,
+                          cudaStream_t st);
+size_t merge_ws_bytes(uint64_t total, int kt);
+cudaError_t launch_merge(const void* a, uint64_t al, const void* b, uint64_t bl, void* out, int kt, void* ws,
+                         cudaStream_t st, int* launches);
+// fill count keys with the largest key under T (tail padding, reading Q3)
+cudaError_t launch_fill_max(void* p, uint64_t count, int kt, cudaStream_t st);
+
+// ----- cross-process device barrier (dist mode) ----------------------------
+struct BarrierArgs {
+    unsigned long long* peer_flags[8];  // flags array of every rank (peer-mapped); slot [rank] written by us
+    unsigned long long* my_flags;       // our own flags array (slot q written by rank q)
+    int rank, world;
+    unsigned long long epoch;
+    unsigned long long timeout_ns;
+    int* err;                            // set to 1 on timeout
+};
+cudaError_t launch_barrier(const BarrierArgs& a, cudaStream_t st);
+
+}  // namespace msort

@@ -1,0 +1,262 @@
+// merge.cu - merge-phase kernels of the P2P sort.
+//
+// Paper: §5.2 "P2P-Based Multi-GPU Sort".
+//   pivot_kernel   Alg.1 Select_Pivot: the leftmost pivot p of
+//                  two concatenated halves A, B of a group (|A| = |B|), read
+//                  through peer pointers ("keys of remote GPUs are accessed via
+//                  P2P memory reads").  One warp runs a 32-ary
+//                  search of the monotone predicate B[i] < A[|A|-1-i] (reading
+//                  Q5): 7 rounds of 64 parallel remote loads instead of ~2*32
+//                  dependent ones.
+//   partition_kernel / merge_kernel
+//                  the local merge of the two sorted runs a GPU holds after a
+//                  swap as a merge-path merge.  In
+//                  the fused exchange mode run b is the PARTNER's block read over
+//                  NVLink inside the merge (the swap and the merge are one
+//                  kernel); in swap mode both runs are local.
+//   fill_kernel    tail padding with the largest key (reading Q3).
+//   barrier_kernel device-side barrier over IPC-mapped flags (dist mode).
+// All comparisons are on T(key) (reading Q1), so floats order by totalOrder.
+#include "common.cuh"
+#include "kernels.h"
+
+namespace msort {
+
+namespace {
+
+// index -> key of the concatenation of equal-size chunks p[first .. first+k)
+template <typename U, bool FLOAT>
+__device__ __forceinline__ U concat_code(const GroupPtrs& g, int first, uint64_t c, uint64_t i) {
+    const uint64_t ch = i / c;
+    return encode<U, FLOAT>(reinterpret_cast<const U*>(g.p[first + ch])[i - ch * c]);
+}
+
+// First index in [lo, hi) where pred is false (pred monotone true->false), or hi.
+// 32-ary search by one warp: every round probes 32 evenly spaced indices.
+template <typename Pred>
+__device__ __forceinline__ uint64_t warp_first_false(uint64_t lo, uint64_t hi, Pred pred) {
+    const int lane = threadIdx.x & 31;
+    while (lo < hi) {
+        const uint64_t step = (hi - lo + 31) / 32;
+        const uint64_t i = lo + uint64_t(lane) * step;
+        const bool valid = i < hi;
+        const bool f = valid && !pred(i);
+        const uint32_t falses = __ballot_sync(0xffffffffu, f);
+        if (falses == 0) {
+            const int nvalid = __popc(__ballot_sync(0xffffffffu, valid));
+            lo = lo + uint64_t(nvalid - 1) * step + 1;
+        } else {
+            const int fl = __ffs(falses) - 1;
+            const uint64_t nhi = lo + uint64_t(fl) * step;
+            if (fl > 0) lo = lo + uint64_t(fl - 1) * step + 1;
+            hi = nhi;
+        }
+    }
+    return lo;
+}
+
+// S4: p = #{i in [0,s) : B[i] < A[s-1-i]} = Alg.1's leftmost pivot.
+// `all` lists the current chunk of every GPU in order; block j handles the
+// group of chunks [j*label, (j+1)*label): A = its left half, B = its right half.
+template <typename U, bool FLOAT>
+__global__ void __launch_bounds__(32) pivot_kernel(GroupPtrs all, int label, uint64_t c, uint64_t* p_out) {
+    const int half = label / 2;
+    const int first = blockIdx.x * label;
+    const uint64_t s = uint64_t(half) * c;
+    const uint64_t p = warp_first_false(0, s, [&](uint64_t i) {
+        const U b = concat_code<U, FLOAT>(all, first + half, c, i);
+        const U a = concat_code<U, FLOAT>(all, first, c, s - 1 - i);
+        return b < a;
+    });
+    if (threadIdx.x == 0) p_out[blockIdx.x] = p;
+}
+
+template <typename U>
+struct MergeCfg;
+template <>
+struct MergeCfg<uint32_t> {
+    static constexpr int kThreads = 256;
+    static constexpr int kIpt = 15;
+};
+template <>
+struct MergeCfg<uint64_t> {
+    static constexpr int kThreads = 256;
+    static constexpr int kIpt = 7;
+};
+
+// Merge-path partition: part[t] = number of a-elements among the first
+// min(t*TILE, total) outputs (a wins ties).  One warp per boundary.
+template <typename U, bool FLOAT>
+__global__ void __launch_bounds__(128) partition_kernel(const U* __restrict__ a, uint64_t al, const U* __restrict__ b,
+                                                        uint64_t bl, uint64_t tile, uint64_t nparts,
+                                                        uint64_t* __restrict__ part) {
+    const uint64_t w = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+    if (w >= nparts) return;
+    const uint64_t total = al + bl;
+    const uint64_t k = w * tile < total ? w * tile : total;
+    const uint64_t lo = k > bl ? k - bl : 0;
+    const uint64_t hi = k < al ? k : al;
+    const uint64_t r = warp_first_false(lo, hi, [&](uint64_t i) {
+        return encode<U, FLOAT>(a[i]) <= encode<U, FLOAT>(b[k - 1 - i]);
+    });
+    if ((threadIdx.x & 31) == 0) part[w] = r;
+}
+
+// Block merge of one output tile: stage both input ranges in smem (as codes),
+// per-thread merge-path split, serial merge of IPT outputs, smem transpose,
+// coalesced store.
+template <typename U, bool FLOAT>
+__global__ void __launch_bounds__(MergeCfg<U>::kThreads) merge_kernel(const U* __restrict__ a, const U* __restrict__ b,
+                                                                      uint64_t al, uint64_t bl, U* __restrict__ out,
+                                                                      const uint64_t* __restrict__ part) {
+    constexpr int THREADS = MergeCfg<U>::kThreads;
+    constexpr int IPT = MergeCfg<U>::kIpt;
+    constexpr int TILE = THREADS * IPT;
+    __shared__ U s[TILE];
+    const int tid = threadIdx.x;
+    const uint64_t total = al + bl;
+    const uint64_t k0 = uint64_t(blockIdx.x) * TILE;
+    const uint64_t k1 = k0 + TILE < total ? k0 + TILE : total;
+    const uint64_t a0 = part[blockIdx.x], a1 = part[blockIdx.x + 1];
+    const uint64_t b0 = k0 - a0, b1 = k1 - a1;
+    const int na = int(a1 - a0), nb = int(b1 - b0), nt = na + nb;
+
+    // load: all IPT loads of a thread are independent (in flight together)
+#pragma unroll
+    for (int r = 0; r < IPT; ++r) {
+        const int j = tid + r * THREADS;
+        if (j < nt) s[j] = encode<U, FLOAT>(j < na ? a[a0 + j] : b[b0 + (j - na)]);
+    }
+    __syncthreads();
+    const U* sa = s;
+    const U* sb = s + na;
+    // this thread's output diagonal
+    const int d0 = min(tid * IPT, nt);
+    int lo = max(0, d0 - nb), hi = min(d0, na);
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (sa[mid] <= sb[d0 - 1 - mid]) lo = mid + 1;
+        else hi = mid;
+    }
+    int ia = lo, ib = d0 - lo;
+    U r[IPT];
+#pragma unroll
+    for (int j = 0; j < IPT; ++j) {
+        const bool takeA = ib >= nb || (ia < na && sa[ia] <= sb[ib]);
+        if (takeA) {
+            r[j] = ia < na ? sa[ia] : U(0);
+            ++ia;
+        } else {
+            r[j] = sb[ib];
+            ++ib;
+        }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < IPT; ++j)
+        if (d0 + j < nt) s[d0 + j] = r[j];
+    __syncthreads();
+#pragma unroll
+    for (int rr = 0; rr < IPT; ++rr) {
+        const int j = tid + rr * THREADS;
+        if (j < nt) out[k0 + j] = decode<U, FLOAT>(s[j]);
+    }
+}
+
+template <typename U, bool FLOAT>
+cudaError_t launch_merge_t(const void* a, uint64_t al, const void* b, uint64_t bl, void* out, void* ws,
+                           cudaStream_t st, int* launches) {
+    constexpr uint64_t TILE = uint64_t(MergeCfg<U>::kThreads) * MergeCfg<U>::kIpt;
+    const uint64_t total = al + bl;
+    const uint64_t tiles = (total + TILE - 1) / TILE;
+    const uint64_t nparts = tiles + 1;
+    uint64_t* part = reinterpret_cast<uint64_t*>(ws);
+    const unsigned pblocks = unsigned((nparts * 32 + 127) / 128);
+    partition_kernel<U, FLOAT><<<pblocks, 128, 0, st>>>((const U*)a, al, (const U*)b, bl, TILE, nparts, part);
+    merge_kernel<U, FLOAT><<<unsigned(tiles), MergeCfg<U>::kThreads, 0, st>>>((const U*)a, (const U*)b, al, bl, (U*)out,
+                                                                            part);
+    if (launches) *launches += 2;
+    return cudaGetLastError();
+}
+
+template <typename U, bool FLOAT>
+__global__ void fill_kernel(U* p, uint64_t count) {
+    const U v = decode<U, FLOAT>(~U(0));
+    for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < count; i += uint64_t(gridDim.x) * blockDim.x)
+        p[i] = v;
+}
+
+__global__ void barrier_kernel(BarrierArgs a) {
+    const int q = threadIdx.x;
+    if (q < a.world && q != a.rank) {
+        // release: everything this GPU wrote before the barrier (earlier
+        // kernels in stream order) is visible to peers that acquire the flag
+        unsigned long long* dst = a.peer_flags[q] + a.rank;
+        asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(dst), "l"(a.epoch) : "memory");
+        const unsigned long long* src = a.my_flags + q;
+        const uint64_t t0 = globaltimer_ns();
+        while (true) {
+            unsigned long long v;
+            asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(src) : "memory");
+            if (v >= a.epoch) break;
+            if (globaltimer_ns() - t0 > a.timeout_ns) {
+                atomicExch(a.err, 1);
+                break;
+            }
+            __nanosleep(256);
+        }
+    }
+    __syncthreads();
+}
+
+}  // namespace
+
+cudaError_t launch_pivots(const GroupPtrs& all, int n_groups, int label, uint64_t c, int kt, uint64_t* d_p,
+                          cudaStream_t st) {
+    switch (kt) {
+        case 0: pivot_kernel<uint32_t, false><<<n_groups, 32, 0, st>>>(all, label, c, d_p); break;
+        case 1: pivot_kernel<uint64_t, false><<<n_groups, 32, 0, st>>>(all, label, c, d_p); break;
+        case 2: pivot_kernel<uint32_t, true><<<n_groups, 32, 0, st>>>(all, label, c, d_p); break;
+        case 3: pivot_kernel<uint64_t, true><<<n_groups, 32, 0, st>>>(all, label, c, d_p); break;
+        default: return cudaErrorInvalidValue;
+    }
+    return cudaGetLastError();
+}
+
+size_t merge_ws_bytes(uint64_t total, int kt) {
+    const uint64_t tile = key_bytes(kt) == 4 ? uint64_t(MergeCfg<uint32_t>::kThreads) * MergeCfg<uint32_t>::kIpt
+                                             : uint64_t(MergeCfg<uint64_t>::kThreads) * MergeCfg<uint64_t>::kIpt;
+    return size_t((total + tile - 1) / tile + 2) * 8 + 256;
+}
+
+cudaError_t launch_merge(const void* a, uint64_t al, const void* b, uint64_t bl, void* out, int kt, void* ws,
+                         cudaStream_t st, int* launches) {
+    if (al + bl == 0) return cudaSuccess;
+    switch (kt) {
+        case 0: return launch_merge_t<uint32_t, false>(a, al, b, bl, out, ws, st, launches);
+        case 1: return launch_merge_t<uint64_t, false>(a, al, b, bl, out, ws, st, launches);
+        case 2: return launch_merge_t<uint32_t, true>(a, al, b, bl, out, ws, st, launches);
+        case 3: return launch_merge_t<uint64_t, true>(a, al, b, bl, out, ws, st, launches);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+cudaError_t launch_fill_max(void* p, uint64_t count, int kt, cudaStream_t st) {
+    if (count == 0) return cudaSuccess;
+    const unsigned blocks = unsigned(count < 256 * 1024 ? (count + 255) / 256 : 1024);
+    switch (kt) {
+        case 0: fill_kernel<uint32_t, false><<<blocks, 256, 0, st>>>((uint32_t*)p, count); break;
+        case 1: fill_kernel<uint64_t, false><<<blocks, 256, 0, st>>>((uint64_t*)p, count); break;
+        case 2: fill_kernel<uint32_t, true><<<blocks, 256, 0, st>>>((uint32_t*)p, count); break;
+        case 3: fill_kernel<uint64_t, true><<<blocks, 256, 0, st>>>((uint64_t*)p, count); break;
+        default: return cudaErrorInvalidValue;
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_barrier(const BarrierArgs& a, cudaStream_t st) {
+    barrier_kernel<<<1, 32, 0, st>>>(a);
+    return cudaGetLastError();
+}
+
+}  // namespace msort

@@ -1,0 +1,1111 @@
+// msort.cpp - C ABI, contexts and the stage scheduler of the P2P sort.
+//
+// Orchestration of PAPER.md §5.2 on B200s:
+//   chunking -> per-GPU radix sort (§5.1, radix.cu) ->
+//   g-1 merge stages of Alg.2: barrier, Alg.1 pivots of every
+//   group (merge.cu), exchange + local merge of each mirrored GPU pair
+//    -> result chunk i = global ranks
+//   [i*c, (i+1)*c).
+// Two execution modes share the plan and the kernels:
+//   * single process (msort_create): one host thread drives g "ranks"; ranks
+//     may be distinct GPUs (peer access over NVLink) or repeated devices
+//     (virtual ranks on one GPU); cross-rank ordering by CUDA events;
+//   * one process per GPU (msort_dist_*): peers' buffers are mapped with CUDA
+//     IPC; cross-rank ordering by a device-side barrier on IPC-mapped flags.
+// Every rank knows every pivot of every stage (each rank computes all of them
+// from peer memory), so the buffer rotation of all ranks is replicated
+// deterministically without extra messages.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <tuple>
+#include <vector>
+
+#include "../../include/msort.h"
+#include "kernels.h"
+
+using namespace msort;
+
+namespace {
+
+thread_local std::string g_last_error;
+
+int set_error(int status, const std::string& msg) {
+    g_last_error = msg;
+    return status;
+}
+
+int cuda_status(cudaError_t e) {
+    switch (e) {
+        case cudaErrorMemoryAllocation: return MSORT_ERR_OUT_OF_MEMORY;
+        case cudaErrorNoDevice:
+        case cudaErrorInsufficientDriver:
+        case cudaErrorInvalidDevice:
+        case cudaErrorPeerAccessUnsupported: return MSORT_ERR_DEVICE;
+        default: return MSORT_ERR_CUDA;
+    }
+}
+
+#define CUDA_TRY(expr)                                                                                  \
+    do {                                                                                                \
+        cudaError_t e_ = (expr);                                                                        \
+        if (e_ != cudaSuccess) {                                                                        \
+            return set_error(cuda_status(e_), std::string(#expr) + " -> " + cudaGetErrorString(e_) +   \
+                                                  " (" + __FILE__ + ":" + std::to_string(__LINE__) + ")"); \
+        }                                                                                               \
+    } while (0)
+
+#define MSORT_TRY(expr)             \
+    do {                            \
+        int s_ = (expr);            \
+        if (s_ != MSORT_OK) return s_; \
+    } while (0)
+
+bool valid_kt(int kt) { return kt >= 0 && kt <= 3; }
+bool valid_g(int g) { return g == 1 || g == 2 || g == 4 || g == 8; }
+
+// ---------------------------------------------------------------------------
+// Plan (host only): Alg.2 stage labels, reading Q7.
+// ---------------------------------------------------------------------------
+void stage_labels(int g, std::vector<int>& out) {
+    if (g < 2) return;
+    if (g == 2) {
+        out.push_back(2);
+        return;
+    }
+    std::vector<int> half;
+    stage_labels(g / 2, half);
+    out.insert(out.end(), half.begin(), half.end());
+    out.push_back(g);
+    out.insert(out.end(), half.begin(), half.end());
+}
+
+struct Exchange {
+    int partner[MSORT_MAX_GPUS];
+    uint64_t x[MSORT_MAX_GPUS];
+    int side[MSORT_MAX_GPUS];
+};
+
+// Reading Q6 (Fig.9).
+void plan_exchange(int g, int label, uint64_t c, const uint64_t* pivots, Exchange& ex) {
+    for (int r = 0; r < g; ++r) {
+        ex.partner[r] = -1;
+        ex.x[r] = 0;
+        ex.side[r] = 0;
+    }
+    for (int j = 0; j < g / label; ++j) {
+        const int lo = j * label, mid = lo + label / 2;
+        const uint64_t p = pivots[j];
+        for (int d = 0; d < label / 2; ++d) {
+            const int L = mid - 1 - d, R = mid + d;
+            const uint64_t dc = uint64_t(d) * c;
+            const uint64_t x = p <= dc ? 0 : std::min<uint64_t>(p - dc, c);
+            ex.partner[L] = R;
+            ex.partner[R] = L;
+            ex.x[L] = ex.x[R] = x;
+            ex.side[L] = 0;
+            ex.side[R] = 1;
+        }
+    }
+}
+
+uint64_t chunk_size(uint64_t n, int g) {
+    const uint64_t c = (n + g - 1) / g;
+    return (c + 3) / 4 * 4;  // reading Q3
+}
+
+// ---------------------------------------------------------------------------
+// Per-rank state
+// ---------------------------------------------------------------------------
+struct Rank {
+    int dev = 0;
+    cudaStream_t st = nullptr;
+    void* buf[3] = {nullptr, nullptr, nullptr};  // B0, B1 (rotating chunk buffers), B2 (swap-mode receive)
+    void* stage = nullptr;                       // chunk staging buffer for host / single-pointer sorts
+    void* rws = nullptr;
+    size_t rws_bytes = 0;
+    void* mws = nullptr;
+    size_t mws_bytes = 0;
+    uint64_t* d_pivot = nullptr;   // [4]
+    uint64_t* h_pivot = nullptr;   // pinned [4]
+    uint32_t* h_trivial = nullptr; // pinned [8]
+    int* d_err = nullptr;          // barrier timeout flag
+    int* h_err = nullptr;          // pinned
+    cudaEvent_t e_begin = nullptr, e_hist = nullptr, e_sorted = nullptr, e_end = nullptr;
+    cudaEvent_t e_h2d0 = nullptr, e_h2d1 = nullptr, e_d2h0 = nullptr, e_d2h1 = nullptr;
+    cudaEvent_t e_pass[8][2] = {};
+    cudaEvent_t e_sync[MSORT_MAX_STAGES + 1] = {};
+    cudaEvent_t e_stage[MSORT_MAX_STAGES][2] = {};
+    cudaEvent_t e_xch[MSORT_MAX_STAGES][2] = {};
+    // per sort
+    void* user = nullptr;
+    int cur = -1;  // -1: user buffer, 0..2: buf[]
+    int passes_run = 0;
+    int pass_ids[8] = {};
+
+    void* ptr(int which) const { return which < 0 ? user : buf[which]; }
+};
+
+struct DeviceGuard {
+    int prev = 0;
+    DeviceGuard() { cudaGetDevice(&prev); }
+    ~DeviceGuard() { cudaSetDevice(prev); }
+};
+
+}  // namespace
+
+struct msort_ctx {
+    int g = 1;
+    int kt = 0;
+    uint64_t cap = 0;  // keys per rank
+    bool dist = false;
+    int rank = 0;      // dist: this process's rank
+    int nlocal = 1;    // ranks driven by this process
+    Rank r[MSORT_MAX_GPUS];
+    // dist mode: buffers and flags of every rank as seen from this process
+    void* peer_buf[MSORT_MAX_GPUS][2] = {};
+    unsigned long long* peer_flags[MSORT_MAX_GPUS] = {};
+    unsigned long long* my_flags = nullptr;
+    unsigned long long epoch = 0;
+    bool imported = false;
+    std::vector<void*> opened;
+    // options
+    int timing = 1;
+    int exchange = 0;
+    int skip_trivial = 1;
+    msort_timings tm{};
+};
+
+namespace {
+
+int alloc_rank(msort_ctx* ctx, Rank& R, bool need_b1, bool need_stage) {
+    const size_t K = key_bytes(ctx->kt);
+    CUDA_TRY(cudaSetDevice(R.dev));
+    CUDA_TRY(cudaStreamCreateWithFlags(&R.st, cudaStreamNonBlocking));
+    const size_t bytes = std::max<size_t>(ctx->cap * K, 256);
+    CUDA_TRY(cudaMalloc(&R.buf[0], bytes));
+    if (need_b1) CUDA_TRY(cudaMalloc(&R.buf[1], bytes));
+    if (need_stage) CUDA_TRY(cudaMalloc(&R.stage, bytes));
+    R.rws_bytes = radix_ws_bytes(ctx->cap, ctx->kt);
+    CUDA_TRY(cudaMalloc(&R.rws, R.rws_bytes));
+    R.mws_bytes = merge_ws_bytes(ctx->cap, ctx->kt);
+    CUDA_TRY(cudaMalloc(&R.mws, R.mws_bytes));
+    CUDA_TRY(cudaMalloc(&R.d_pivot, 8 * sizeof(uint64_t)));
+    CUDA_TRY(cudaMalloc(&R.d_err, sizeof(int)));
+    CUDA_TRY(cudaMemset(R.d_err, 0, sizeof(int)));
+    CUDA_TRY(cudaMallocHost(&R.h_pivot, 8 * sizeof(uint64_t)));
+    CUDA_TRY(cudaMallocHost(&R.h_trivial, 8 * sizeof(uint32_t)));
+    CUDA_TRY(cudaMallocHost(&R.h_err, sizeof(int)));
+    *R.h_err = 0;
+    cudaEvent_t* evs[] = {&R.e_begin, &R.e_hist, &R.e_sorted, &R.e_end, &R.e_h2d0, &R.e_h2d1, &R.e_d2h0, &R.e_d2h1};
+    for (auto* e : evs) CUDA_TRY(cudaEventCreate(e));
+    for (auto& pe : R.e_pass)
+        for (auto& e : pe) CUDA_TRY(cudaEventCreate(&e));
+    for (auto& e : R.e_sync) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    for (auto& se : R.e_stage)
+        for (auto& e : se) CUDA_TRY(cudaEventCreate(&e));
+    for (auto& xe : R.e_xch)
+        for (auto& e : xe) CUDA_TRY(cudaEventCreate(&e));
+    return MSORT_OK;
+}
+
+void free_rank(Rank& R) {
+    if (!R.st) return;
+    cudaSetDevice(R.dev);
+    cudaStreamSynchronize(R.st);
+    for (void* p : R.buf)
+        if (p) cudaFree(p);
+    if (R.stage) cudaFree(R.stage);
+    if (R.rws) cudaFree(R.rws);
+    if (R.mws) cudaFree(R.mws);
+    if (R.d_pivot) cudaFree(R.d_pivot);
+    if (R.d_err) cudaFree(R.d_err);
+    if (R.h_pivot) cudaFreeHost(R.h_pivot);
+    if (R.h_trivial) cudaFreeHost(R.h_trivial);
+    if (R.h_err) cudaFreeHost(R.h_err);
+    cudaEvent_t evs[] = {R.e_begin, R.e_hist, R.e_sorted, R.e_end, R.e_h2d0, R.e_h2d1, R.e_d2h0, R.e_d2h1};
+    for (auto e : evs)
+        if (e) cudaEventDestroy(e);
+    for (auto& pe : R.e_pass)
+        for (auto e : pe)
+            if (e) cudaEventDestroy(e);
+    for (auto e : R.e_sync)
+        if (e) cudaEventDestroy(e);
+    for (auto& se : R.e_stage)
+        for (auto e : se)
+            if (e) cudaEventDestroy(e);
+    for (auto& xe : R.e_xch)
+        for (auto e : xe)
+            if (e) cudaEventDestroy(e);
+    cudaStreamDestroy(R.st);
+    R = Rank();
+}
+
+float elapsed(cudaEvent_t a, cudaEvent_t b) {
+    float ms = 0.f;
+    if (cudaEventElapsedTime(&ms, a, b) != cudaSuccess) {
+        cudaGetLastError();
+        return 0.f;
+    }
+    return ms;
+}
+
+// --- radix phase (S1-S3) -----------------------------------------------------
+
+int radix_begin(msort_ctx* ctx, Rank& R, const void* src, uint64_t c) {
+    CUDA_TRY(cudaSetDevice(R.dev));
+    RadixWs ws = radix_ws_layout(R.rws, c, ctx->kt);
+    CUDA_TRY(radix_prologue(src, c, ctx->kt, ws, R.st));
+    ctx->tm.kernel_launches += 2;
+    if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_hist, R.st));
+    if (ctx->skip_trivial) CUDA_TRY(cudaMemcpyAsync(R.h_trivial, ws.trivial, 8 * sizeof(uint32_t), cudaMemcpyDeviceToHost, R.st));
+    return MSORT_OK;
+}
+
+// src -> dst through tmp; an even number of executed passes, so the last write
+// lands in dst and no pass reads and writes the same buffer.
+int radix_passes(msort_ctx* ctx, Rank& R, const void* src, void* dst, void* tmp, uint64_t c) {
+    CUDA_TRY(cudaSetDevice(R.dev));
+    const int P = num_passes(ctx->kt);
+    RadixWs ws = radix_ws_layout(R.rws, c, ctx->kt);
+    bool run[8];
+    int nrun = 0;
+    for (int p = 0; p < P; ++p) {
+        run[p] = !(ctx->skip_trivial && R.h_trivial[p]);
+        nrun += run[p];
+    }
+    if (nrun % 2) {  // un-skip one trivial pass (an identity permutation) to keep the parity
+        for (int p = 0; p < P; ++p)
+            if (!run[p]) {
+                run[p] = true;
+                ++nrun;
+                break;
+            }
+    }
+    R.passes_run = 0;
+    for (int p = 0; p < P; ++p)
+        if (run[p]) R.pass_ids[R.passes_run++] = p;
+    const int E = R.passes_run;
+    if (E == 0) {
+        if (src != dst) CUDA_TRY(cudaMemcpyAsync(dst, src, c * key_bytes(ctx->kt), cudaMemcpyDeviceToDevice, R.st));
+        return MSORT_OK;
+    }
+    const void* in = src;
+    for (int j = 0; j < E; ++j) {
+        void* out = ((E - 1 - j) % 2 == 0) ? dst : tmp;
+        const int flags = (j == 0 ? 1 : 0) | (j == E - 1 ? 2 : 0);
+        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_pass[j][0], R.st));
+        CUDA_TRY(launch_onesweep(in, out, c, ctx->kt, R.pass_ids[j], flags, ws, ws.base + R.pass_ids[j] * 256, R.st));
+        ctx->tm.kernel_launches += 1;
+        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_pass[j][1], R.st));
+        in = out;
+    }
+    return MSORT_OK;
+}
+
+// --- merge phase (S4-S7) ------------------------------------------------------
+
+// Launch this rank's exchange+merge for one stage. `own` is its current chunk,
+// `peer` the partner's current chunk (peer pointer); returns the new cur index.
+int launch_exchange(msort_ctx* ctx, Rank& R, int stage, bool last, uint64_t c, uint64_t x, int side, const void* own,
+                    const void* peer, int& new_cur) {
+    const size_t K = key_bytes(ctx->kt);
+    const char* ownb = static_cast<const char*>(own);
+    const char* peerb = static_cast<const char*>(peer);
+    new_cur = R.cur;
+    if (x == 0) return MSORT_OK;  // Alg.2 line 7 / reading Q8
+    const int out_idx = last ? -1 : (R.cur == 0 ? 1 : 0);
+    void* out = R.ptr(out_idx);
+    if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[stage][0], R.st));
+    if (x == c) {
+        // the whole chunk moves: a pure P2P copy (one sorted run, reading Q8)
+        CUDA_TRY(cudaMemcpyAsync(out, peer, c * K, cudaMemcpyDefault, R.st));
+    } else if (ctx->exchange == 0) {
+        // fused: the merge kernel reads the partner's block over NVLink
+        if (side == 0)
+            CUDA_TRY(launch_merge(ownb, c - x, peerb, x, out, ctx->kt, R.mws, R.st, &ctx->tm.kernel_launches));
+        else
+            CUDA_TRY(launch_merge(peerb + (c - x) * K, x, ownb + x * K, c - x, out, ctx->kt, R.mws, R.st, &ctx->tm.kernel_launches));
+    } else {
+        // swap (P2P copy into the receive buffer), then local merge
+        char* recv = static_cast<char*>(R.buf[2]);
+        if (side == 0) {
+            CUDA_TRY(cudaMemcpyAsync(recv, peerb, x * K, cudaMemcpyDefault, R.st));
+            CUDA_TRY(launch_merge(ownb, c - x, recv, x, out, ctx->kt, R.mws, R.st, &ctx->tm.kernel_launches));
+        } else {
+            CUDA_TRY(cudaMemcpyAsync(recv, peerb + (c - x) * K, x * K, cudaMemcpyDefault, R.st));
+            CUDA_TRY(launch_merge(recv, x, ownb + x * K, c - x, out, ctx->kt, R.mws, R.st, &ctx->tm.kernel_launches));
+        }
+    }
+    if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[stage][1], R.st));
+    new_cur = out_idx;
+    return MSORT_OK;
+}
+
+int check_c(msort_ctx* ctx, uint64_t c) {
+    if (c > ctx->cap) return set_error(MSORT_ERR_INVALID_ARGUMENT, "keys per GPU exceed the context capacity");
+    if (c >= (1ull << 32)) return set_error(MSORT_ERR_INVALID_ARGUMENT, "keys per GPU must be < 2^32");
+    return MSORT_OK;
+}
+
+void reset_timings(msort_ctx* ctx, uint64_t c) {
+    ctx->tm = msort_timings{};
+    ctx->tm.n_gpus = ctx->g;
+    ctx->tm.keys_per_gpu = c;
+    ctx->tm.passes_total = num_passes(ctx->kt);
+}
+
+// Single-process device-resident sort of r[i].user (c keys each).
+int sort_device_local(msort_ctx* ctx, uint64_t c) {
+    const int g = ctx->g;
+    std::vector<int> labels;
+    stage_labels(g, labels);
+    for (int i = 0; i < g; ++i) {
+        Rank& R = ctx->r[i];
+        CUDA_TRY(cudaSetDevice(R.dev));
+        CUDA_TRY(cudaEventRecord(R.e_begin, R.st));
+        R.cur = -1;
+        MSORT_TRY(radix_begin(ctx, R, R.user, c));
+    }
+    if (ctx->skip_trivial)
+        for (int i = 0; i < g; ++i) CUDA_TRY(cudaStreamSynchronize(ctx->r[i].st));
+    for (int i = 0; i < g; ++i) {
+        Rank& R = ctx->r[i];
+        if (g == 1) {
+            MSORT_TRY(radix_passes(ctx, R, R.user, R.user, R.buf[0], c));
+            R.cur = -1;
+        } else {
+            MSORT_TRY(radix_passes(ctx, R, R.user, R.buf[1], R.buf[0], c));
+            R.cur = 1;
+        }
+        CUDA_TRY(cudaEventRecord(R.e_sorted, R.st));
+    }
+    const int S = int(labels.size());
+    ctx->tm.n_stages = S;
+    for (int s = 0; s < S; ++s) {
+        const int label = labels[s];
+        const bool last = s == S - 1;
+        // barrier: every rank's stream waits for every other rank's previous stage
+        for (int i = 0; i < g; ++i) {
+            CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
+            CUDA_TRY(cudaEventRecord(ctx->r[i].e_sync[s], ctx->r[i].st));
+        }
+        for (int i = 0; i < g; ++i) {
+            Rank& R = ctx->r[i];
+            CUDA_TRY(cudaSetDevice(R.dev));
+            for (int q = 0; q < g; ++q)
+                if (q != i) CUDA_TRY(cudaStreamWaitEvent(R.st, ctx->r[q].e_sync[s], 0));
+            if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[s][0], R.st));
+        }
+        // S4: all pivots of the stage in one launch on rank 0 (peer reads)
+        GroupPtrs all{};
+        for (int i = 0; i < g; ++i) all.p[i] = ctx->r[i].ptr(ctx->r[i].cur);
+        Rank& R0 = ctx->r[0];
+        CUDA_TRY(cudaSetDevice(R0.dev));
+        const int ngroups = g / label;
+        CUDA_TRY(launch_pivots(all, ngroups, label, c, ctx->kt, R0.d_pivot, R0.st));
+        ctx->tm.kernel_launches += 1;
+        CUDA_TRY(cudaMemcpyAsync(R0.h_pivot, R0.d_pivot, ngroups * sizeof(uint64_t), cudaMemcpyDeviceToHost, R0.st));
+        CUDA_TRY(cudaStreamSynchronize(R0.st));
+        uint64_t piv[MSORT_MAX_GPUS / 2] = {};
+        for (int j = 0; j < ngroups; ++j) piv[j] = R0.h_pivot[j];
+        Exchange ex;
+        plan_exchange(g, label, c, piv, ex);
+        ctx->tm.stage_label[s] = label;
+        for (int j = 0; j < ngroups; ++j) ctx->tm.stage_pivot[s][j] = piv[j];
+        uint64_t mx = 0, sum = 0;
+        for (int i = 0; i < g; ++i) {
+            mx = std::max(mx, ex.x[i]);
+            if (ex.side[i] == 0) sum += ex.x[i];
+        }
+        ctx->tm.stage_max_x[s] = mx;
+        ctx->tm.stage_keys_exchanged[s] = sum;
+        // S5+S6 on every rank
+        int new_cur[MSORT_MAX_GPUS];
+        for (int i = 0; i < g; ++i) {
+            Rank& R = ctx->r[i];
+            CUDA_TRY(cudaSetDevice(R.dev));
+            const void* own = R.ptr(R.cur);
+            const void* peer = ex.partner[i] >= 0 ? ctx->r[ex.partner[i]].ptr(ctx->r[ex.partner[i]].cur) : nullptr;
+            MSORT_TRY(launch_exchange(ctx, R, s, last, c, ex.x[i], ex.side[i], own, peer, new_cur[i]));
+            if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[s][1], R.st));
+        }
+        for (int i = 0; i < g; ++i) ctx->r[i].cur = new_cur[i];
+    }
+    for (int i = 0; i < g; ++i) {
+        Rank& R = ctx->r[i];
+        CUDA_TRY(cudaSetDevice(R.dev));
+        if (R.cur != -1)
+            CUDA_TRY(cudaMemcpyAsync(R.user, R.ptr(R.cur), c * key_bytes(ctx->kt), cudaMemcpyDeviceToDevice, R.st));
+        CUDA_TRY(cudaEventRecord(R.e_end, R.st));
+    }
+    return MSORT_OK;
+}
+
+// Fill timings after all events completed.
+void collect_timings(msort_ctx* ctx, int nranks, const uint64_t* xs_by_stage_rank = nullptr) {
+    (void)xs_by_stage_rank;
+    msort_timings& t = ctx->tm;
+    for (int i = 0; i < nranks; ++i) {
+        Rank& R = ctx->r[i];
+        cudaSetDevice(R.dev);
+        t.sort_ms = std::max(t.sort_ms, double(elapsed(R.e_begin, R.e_sorted)));
+        t.merge_ms = std::max(t.merge_ms, double(elapsed(R.e_sorted, R.e_end)));
+        if (ctx->timing) {
+            t.hist_ms = std::max(t.hist_ms, double(elapsed(R.e_begin, R.e_hist)));
+            double ps = 0;
+            for (int j = 0; j < R.passes_run; ++j) ps += elapsed(R.e_pass[j][0], R.e_pass[j][1]);
+            t.pass_ms_sum = std::max(t.pass_ms_sum, ps);
+            for (int s = 0; s < t.n_stages; ++s) {
+                t.stage_ms[s] = std::max(t.stage_ms[s], double(elapsed(R.e_stage[s][0], R.e_stage[s][1])));
+            }
+        }
+        t.passes_run = std::max(t.passes_run, R.passes_run);
+    }
+}
+
+// exchange timings need to know which ranks recorded e_xch in which stage
+struct XchLog {
+    bool rec[MSORT_MAX_STAGES][MSORT_MAX_GPUS] = {};
+};
+
+std::mutex g_cache_mu;
+std::map<std::tuple<int, int, int>, msort_ctx*> g_cache;  // (g, first device, kt) -> ctx
+
+}  // namespace
+
+// ===========================================================================
+// C ABI
+// ===========================================================================
+extern "C" {
+
+const char* msort_status_string(int status) {
+    switch (status) {
+        case MSORT_OK: return "MSORT_OK";
+        case MSORT_ERR_INVALID_ARGUMENT: return "MSORT_ERR_INVALID_ARGUMENT";
+        case MSORT_ERR_DEVICE: return "MSORT_ERR_DEVICE";
+        case MSORT_ERR_OUT_OF_MEMORY: return "MSORT_ERR_OUT_OF_MEMORY";
+        case MSORT_ERR_CUDA: return "MSORT_ERR_CUDA";
+        case MSORT_ERR_NCCL: return "MSORT_ERR_NCCL";
+        case MSORT_ERR_INTERNAL: return "MSORT_ERR_INTERNAL";
+        case MSORT_ERR_TIMEOUT: return "MSORT_ERR_TIMEOUT";
+        default: return "MSORT_ERR_UNKNOWN";
+    }
+}
+
+const char* msort_last_error(void) { return g_last_error.c_str(); }
+
+int msort_version(void) { return 100; }
+
+// --- plan ---------------------------------------------------------------------
+
+int msort_plan_num_stages(int g) {
+    if (!valid_g(g) && g != 16) return -1;
+    return g - 1;
+}
+
+int msort_plan_stage(int g, int s, int* label) {
+    if ((!valid_g(g) && g != 16) || !label) return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad g or label");
+    std::vector<int> labels;
+    stage_labels(g, labels);
+    if (s < 0 || s >= int(labels.size())) return set_error(MSORT_ERR_INVALID_ARGUMENT, "stage out of range");
+    *label = labels[s];
+    return MSORT_OK;
+}
+
+int msort_plan_exchange(int g, int s, uint64_t c, const uint64_t* pivots, int* partner, uint64_t* x, int* side) {
+    int label = 0;
+    if (g > MSORT_MAX_GPUS) return set_error(MSORT_ERR_INVALID_ARGUMENT, "g > 8");
+    MSORT_TRY(msort_plan_stage(g, s, &label));
+    if (!pivots || !partner || !x || !side) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL output");
+    Exchange ex;
+    plan_exchange(g, label, c, pivots, ex);
+    for (int r = 0; r < g; ++r) {
+        partner[r] = ex.partner[r];
+        x[r] = ex.x[r];
+        side[r] = ex.side[r];
+    }
+    return MSORT_OK;
+}
+
+// --- step-level ---------------------------------------------------------------
+
+uint64_t msort_radix_workspace_bytes(uint64_t n, int key_type) {
+    if (!valid_kt(key_type)) return 0;
+    return radix_ws_bytes(n, key_type);
+}
+
+int msort_step_histogram(const void* d_keys, uint64_t n, int key_type, uint32_t* d_hist, void* stream) {
+    if (!valid_kt(key_type) || !d_hist || (n && !d_keys)) return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad argument");
+    if (n >= (1ull << 32)) return set_error(MSORT_ERR_INVALID_ARGUMENT, "n must be < 2^32");
+    CUDA_TRY(launch_histogram(d_keys, n, key_type, d_hist, static_cast<cudaStream_t>(stream)));
+    return MSORT_OK;
+}
+
+int msort_step_radix_pass(const void* d_in, void* d_out, uint64_t n, int key_type, int pass, const uint32_t* d_hist,
+                          int flags, void* d_ws, uint64_t ws_bytes, void* stream) {
+    if (!valid_kt(key_type) || pass < 0 || pass >= num_passes(key_type) || !d_hist || (n && (!d_in || !d_out)))
+        return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad argument");
+    if (n >= (1ull << 32)) return set_error(MSORT_ERR_INVALID_ARGUMENT, "n must be < 2^32");
+    if (d_in == d_out) return set_error(MSORT_ERR_INVALID_ARGUMENT, "a pass is out of place");
+    if (ws_bytes < radix_ws_bytes(n, key_type) || !d_ws) return set_error(MSORT_ERR_INVALID_ARGUMENT, "workspace too small");
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    RadixWs ws = radix_ws_layout(d_ws, n, key_type);
+    CUDA_TRY(cudaMemsetAsync(ws.counters, 0, ws.head_bytes + size_t(ws.tiles) * 256 * 8, st));
+    CUDA_TRY(launch_scan(d_hist, ws.base, ws.trivial, n, key_type, st));
+    CUDA_TRY(launch_onesweep(d_in, d_out, n, key_type, pass, flags & 3, ws, ws.base + pass * 256, st));
+    return MSORT_OK;
+}
+
+int msort_radix_sort(void* d_keys, void* d_aux, uint64_t n, int key_type, void* d_ws, uint64_t ws_bytes, void* stream) {
+    if (!valid_kt(key_type) || (n && (!d_keys || !d_aux))) return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad argument");
+    if (n >= (1ull << 32)) return set_error(MSORT_ERR_INVALID_ARGUMENT, "n must be < 2^32");
+    if (n <= 1) return MSORT_OK;
+    if (ws_bytes < radix_ws_bytes(n, key_type) || !d_ws) return set_error(MSORT_ERR_INVALID_ARGUMENT, "workspace too small");
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    RadixWs ws = radix_ws_layout(d_ws, n, key_type);
+    CUDA_TRY(radix_prologue(d_keys, n, key_type, ws, st));
+    const int P = num_passes(key_type);
+    for (int p = 0; p < P; ++p) {
+        const void* in = (p % 2 == 0) ? d_keys : d_aux;
+        void* out = (p % 2 == 0) ? d_aux : d_keys;
+        const int flags = (p == 0 ? 1 : 0) | (p == P - 1 ? 2 : 0);
+        CUDA_TRY(launch_onesweep(in, out, n, key_type, p, flags, ws, ws.base + p * 256, st));
+    }
+    return MSORT_OK;
+}
+
+int msort_step_pivot(const void* const* d_chunks, int n_chunks, uint64_t c, int key_type, uint64_t* d_pivot,
+                     void* stream) {
+    if (!valid_kt(key_type) || !d_chunks || !d_pivot || n_chunks < 2 || n_chunks > MSORT_MAX_GPUS || n_chunks % 2)
+        return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad argument");
+    GroupPtrs all{};
+    for (int i = 0; i < n_chunks; ++i) all.p[i] = d_chunks[i];
+    if (c == 0) {
+        CUDA_TRY(cudaMemsetAsync(d_pivot, 0, 8, static_cast<cudaStream_t>(stream)));
+        return MSORT_OK;
+    }
+    CUDA_TRY(launch_pivots(all, 1, n_chunks, c, key_type, d_pivot, static_cast<cudaStream_t>(stream)));
+    return MSORT_OK;
+}
+
+uint64_t msort_merge_workspace_bytes(uint64_t total, int key_type) {
+    if (!valid_kt(key_type)) return 0;
+    return merge_ws_bytes(total, key_type);
+}
+
+int msort_step_merge(const void* d_a, uint64_t a_len, const void* d_b, uint64_t b_len, void* d_out, int key_type,
+                     void* d_ws, uint64_t ws_bytes, void* stream) {
+    if (!valid_kt(key_type) || (a_len && !d_a) || (b_len && !d_b) || (a_len + b_len && !d_out))
+        return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad argument");
+    if (ws_bytes < merge_ws_bytes(a_len + b_len, key_type) || !d_ws)
+        return set_error(MSORT_ERR_INVALID_ARGUMENT, "workspace too small");
+    CUDA_TRY(launch_merge(d_a, a_len, d_b, b_len, d_out, key_type, d_ws, static_cast<cudaStream_t>(stream), nullptr));
+    return MSORT_OK;
+}
+
+// --- context ------------------------------------------------------------------
+
+int msort_create(msort_ctx** out, int n_gpus, const int* device_ids, uint64_t max_keys, int key_type) {
+    if (!out || !valid_g(n_gpus) || !valid_kt(key_type)) return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad argument");
+    *out = nullptr;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        return set_error(MSORT_ERR_DEVICE, "no CUDA device");
+    }
+    DeviceGuard guard;
+    auto ctx = std::make_unique<msort_ctx>();
+    ctx->g = n_gpus;
+    ctx->kt = key_type;
+    ctx->nlocal = n_gpus;
+    ctx->cap = chunk_size(std::max<uint64_t>(max_keys, 4), n_gpus);
+    if (ctx->cap >= (1ull << 32)) return set_error(MSORT_ERR_INVALID_ARGUMENT, "keys per GPU must be < 2^32");
+    for (int i = 0; i < n_gpus; ++i) {
+        const int d = device_ids ? device_ids[i] : i;
+        if (d < 0 || d >= ndev) return set_error(MSORT_ERR_DEVICE, "device id out of range / too few GPUs");
+        ctx->r[i].dev = d;
+    }
+    // peer access between distinct devices (P2P reads and copies over NVLink)
+    for (int i = 0; i < n_gpus; ++i)
+        for (int j = 0; j < n_gpus; ++j) {
+            const int a = ctx->r[i].dev, b = ctx->r[j].dev;
+            if (a == b) continue;
+            int can = 0;
+            CUDA_TRY(cudaDeviceCanAccessPeer(&can, a, b));
+            if (!can) return set_error(MSORT_ERR_DEVICE, "no peer access between GPUs");
+            CUDA_TRY(cudaSetDevice(a));
+            cudaError_t e = cudaDeviceEnablePeerAccess(b, 0);
+            if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+            else if (e != cudaSuccess) return set_error(MSORT_ERR_DEVICE, cudaGetErrorString(e));
+        }
+    for (int i = 0; i < n_gpus; ++i) {
+        int s = alloc_rank(ctx.get(), ctx->r[i], n_gpus > 1, true);
+        if (s != MSORT_OK) {
+            for (int j = 0; j <= i; ++j) free_rank(ctx->r[j]);
+            return s;
+        }
+    }
+    *out = ctx.release();
+    return MSORT_OK;
+}
+
+int msort_destroy(msort_ctx* ctx) {
+    if (!ctx) return MSORT_OK;
+    DeviceGuard guard;
+    if (ctx->dist) {
+        cudaSetDevice(ctx->r[0].dev);
+        for (void* p : ctx->opened) cudaIpcCloseMemHandle(p);
+        if (ctx->my_flags) cudaFree(ctx->my_flags);
+    }
+    for (int i = 0; i < ctx->nlocal; ++i) free_rank(ctx->r[i]);
+    delete ctx;
+    return MSORT_OK;
+}
+
+int msort_set_option(msort_ctx* ctx, int option, int64_t value) {
+    if (!ctx) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL ctx");
+    DeviceGuard guard;
+    switch (option) {
+        case MSORT_OPT_TIMING: ctx->timing = value ? 1 : 0; return MSORT_OK;
+        case MSORT_OPT_SKIP_TRIVIAL: ctx->skip_trivial = value ? 1 : 0; return MSORT_OK;
+        case MSORT_OPT_EXCHANGE:
+            if (value != 0 && value != 1) return set_error(MSORT_ERR_INVALID_ARGUMENT, "exchange mode 0 or 1");
+            if (value == 1)
+                for (int i = 0; i < ctx->nlocal; ++i)
+                    if (!ctx->r[i].buf[2]) {
+                        CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
+                        CUDA_TRY(cudaMalloc(&ctx->r[i].buf[2], std::max<size_t>(ctx->cap * key_bytes(ctx->kt), 256)));
+                    }
+            ctx->exchange = int(value);
+            return MSORT_OK;
+        default: return set_error(MSORT_ERR_INVALID_ARGUMENT, "unknown option");
+    }
+}
+
+int msort_get_timings(const msort_ctx* ctx, msort_timings* out) {
+    if (!ctx || !out) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL argument");
+    *out = ctx->tm;
+    return MSORT_OK;
+}
+
+static int finish_local(msort_ctx* ctx) {
+    for (int i = 0; i < ctx->g; ++i) {
+        CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
+        CUDA_TRY(cudaEventSynchronize(ctx->r[i].e_end));
+    }
+    return MSORT_OK;
+}
+
+static void collect_exchange_timings(msort_ctx* ctx) {
+    if (!ctx->timing) return;
+    // e_xch events are recorded only on ranks that exchanged; query each and
+    // keep the ones that completed (cudaEventElapsedTime fails on unrecorded)
+    for (int s = 0; s < ctx->tm.n_stages; ++s) {
+        double mx = 0;
+        for (int i = 0; i < ctx->nlocal; ++i) {
+            Rank& R = ctx->r[i];
+            cudaSetDevice(R.dev);
+            float ms = 0.f;
+            if (cudaEventElapsedTime(&ms, R.e_xch[s][0], R.e_xch[s][1]) == cudaSuccess) mx = std::max(mx, double(ms));
+            else cudaGetLastError();
+        }
+        ctx->tm.stage_exchange_ms[s] = mx;
+    }
+}
+
+int msort_sort_device(msort_ctx* ctx, void* const* chunks, uint64_t keys_per_gpu, void* const* streams) {
+    if (!ctx || ctx->dist) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL or dist ctx");
+    if (keys_per_gpu && !chunks) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL chunks");
+    MSORT_TRY(check_c(ctx, keys_per_gpu));
+    if (keys_per_gpu == 0 || (ctx->g == 1 && keys_per_gpu <= 1)) return MSORT_OK;
+    DeviceGuard guard;
+    reset_timings(ctx, keys_per_gpu);
+    // re-create per-sort exchange events so stale records never alias
+    for (int i = 0; i < ctx->g; ++i) {
+        if (!chunks[i]) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL chunk");
+        Rank& R = ctx->r[i];
+        R.user = chunks[i];
+        CUDA_TRY(cudaSetDevice(R.dev));
+        for (int s = 0; s < MSORT_MAX_STAGES; ++s)
+            for (auto& e : R.e_xch[s]) {
+                CUDA_TRY(cudaEventDestroy(e));
+                CUDA_TRY(cudaEventCreate(&e));
+            }
+        if (streams && streams[i]) {
+            CUDA_TRY(cudaEventRecord(R.e_sync[MSORT_MAX_STAGES], static_cast<cudaStream_t>(streams[i])));
+            CUDA_TRY(cudaStreamWaitEvent(R.st, R.e_sync[MSORT_MAX_STAGES], 0));
+        }
+    }
+    MSORT_TRY(sort_device_local(ctx, keys_per_gpu));
+    for (int i = 0; i < ctx->g; ++i)
+        if (streams && streams[i]) {
+            CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
+            CUDA_TRY(cudaStreamWaitEvent(static_cast<cudaStream_t>(streams[i]), ctx->r[i].e_end, 0));
+        }
+    MSORT_TRY(finish_local(ctx));
+    collect_timings(ctx, ctx->g);
+    collect_exchange_timings(ctx);
+    ctx->tm.total_ms = ctx->tm.sort_ms + ctx->tm.merge_ms;
+    return MSORT_OK;
+}
+
+int msort_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n) {
+    if (!ctx || ctx->dist) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL or dist ctx");
+    if (n && !host_keys) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL keys");
+    if (n <= 1) return MSORT_OK;
+    const int g = ctx->g;
+    const uint64_t c = chunk_size(n, g);
+    MSORT_TRY(check_c(ctx, c));
+    DeviceGuard guard;
+    reset_timings(ctx, c);
+    const size_t K = key_bytes(ctx->kt);
+    char* host = static_cast<char*>(host_keys);
+    for (int i = 0; i < g; ++i) {
+        Rank& R = ctx->r[i];
+        CUDA_TRY(cudaSetDevice(R.dev));
+        for (int s = 0; s < MSORT_MAX_STAGES; ++s)
+            for (auto& e : R.e_xch[s]) {
+                CUDA_TRY(cudaEventDestroy(e));
+                CUDA_TRY(cudaEventCreate(&e));
+            }
+        R.user = R.stage;
+        const uint64_t lo = std::min<uint64_t>(n, uint64_t(i) * c);
+        const uint64_t cnt = std::min<uint64_t>(n - lo, c);
+        CUDA_TRY(cudaEventRecord(R.e_h2d0, R.st));
+        if (cnt) CUDA_TRY(cudaMemcpyAsync(R.stage, host + lo * K, cnt * K, cudaMemcpyHostToDevice, R.st));
+        CUDA_TRY(launch_fill_max(static_cast<char*>(R.stage) + cnt * K, c - cnt, ctx->kt, R.st));
+        if (c > cnt) ctx->tm.kernel_launches += 1;
+        CUDA_TRY(cudaEventRecord(R.e_h2d1, R.st));
+    }
+    MSORT_TRY(sort_device_local(ctx, c));
+    for (int i = 0; i < g; ++i) {
+        Rank& R = ctx->r[i];
+        CUDA_TRY(cudaSetDevice(R.dev));
+        const uint64_t lo = std::min<uint64_t>(n, uint64_t(i) * c);
+        const uint64_t cnt = std::min<uint64_t>(n - lo, c);
+        CUDA_TRY(cudaEventRecord(R.e_d2h0, R.st));
+        if (cnt) CUDA_TRY(cudaMemcpyAsync(host + lo * K, R.stage, cnt * K, cudaMemcpyDeviceToHost, R.st));
+        CUDA_TRY(cudaEventRecord(R.e_d2h1, R.st));
+    }
+    for (int i = 0; i < g; ++i) {
+        CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
+        CUDA_TRY(cudaEventSynchronize(ctx->r[i].e_d2h1));
+    }
+    collect_timings(ctx, g);
+    collect_exchange_timings(ctx);
+    for (int i = 0; i < g; ++i) {
+        Rank& R = ctx->r[i];
+        cudaSetDevice(R.dev);
+        ctx->tm.h2d_ms = std::max(ctx->tm.h2d_ms, double(elapsed(R.e_h2d0, R.e_h2d1)));
+        ctx->tm.d2h_ms = std::max(ctx->tm.d2h_ms, double(elapsed(R.e_d2h0, R.e_d2h1)));
+        ctx->tm.total_ms = std::max(ctx->tm.total_ms, double(elapsed(R.e_h2d0, R.e_d2h1)));
+    }
+    return MSORT_OK;
+}
+
+int msort_sort(void* keys, uint64_t n, int key_type, int n_gpus, void* stream) {
+    if (!valid_kt(key_type) || !valid_g(n_gpus)) return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad key_type or n_gpus");
+    if (n <= 1) return MSORT_OK;
+    if (!keys) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL keys");
+    DeviceGuard guard;
+    cudaPointerAttributes attr{};
+    cudaError_t ae = cudaPointerGetAttributes(&attr, keys);
+    if (ae != cudaSuccess) {
+        cudaGetLastError();
+        attr.type = cudaMemoryTypeUnregistered;
+    }
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev < n_gpus) {
+        cudaGetLastError();
+        return set_error(MSORT_ERR_DEVICE, "too few CUDA devices");
+    }
+    const bool on_device = attr.type == cudaMemoryTypeDevice || attr.type == cudaMemoryTypeManaged;
+    const int first_dev = on_device && n_gpus == 1 ? attr.device : 0;
+    std::lock_guard<std::mutex> lock(g_cache_mu);
+    auto key = std::make_tuple(n_gpus, first_dev, key_type);
+    msort_ctx* ctx = g_cache.count(key) ? g_cache[key] : nullptr;
+    const uint64_t c = chunk_size(n, n_gpus);
+    if (ctx && ctx->cap < c) {
+        msort_destroy(ctx);
+        ctx = nullptr;
+    }
+    if (!ctx) {
+        std::vector<int> devs(n_gpus);
+        for (int i = 0; i < n_gpus; ++i) devs[i] = first_dev + i;
+        MSORT_TRY(msort_create(&ctx, n_gpus, devs.data(), n, key_type));
+        g_cache[key] = ctx;
+    }
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    if (!on_device) {
+        CUDA_TRY(cudaStreamSynchronize(st));
+        return msort_sort_host(ctx, keys, n);
+    }
+    if (n_gpus == 1) {
+        void* chunks[1] = {keys};
+        void* streams[1] = {stream};
+        return msort_sort_device(ctx, chunks, n, stream ? streams : nullptr);
+    }
+    // device pointer, several GPUs: distribute into the per-GPU staging chunks
+    CUDA_TRY(cudaStreamSynchronize(st));
+    const size_t K = key_bytes(key_type);
+    char* src = static_cast<char*>(keys);
+    std::vector<void*> chunks(n_gpus);
+    for (int i = 0; i < n_gpus; ++i) {
+        Rank& R = ctx->r[i];
+        CUDA_TRY(cudaSetDevice(R.dev));
+        const uint64_t lo = std::min<uint64_t>(n, uint64_t(i) * c);
+        const uint64_t cnt = std::min<uint64_t>(n - lo, c);
+        if (cnt) CUDA_TRY(cudaMemcpyAsync(R.stage, src + lo * K, cnt * K, cudaMemcpyDefault, R.st));
+        CUDA_TRY(launch_fill_max(static_cast<char*>(R.stage) + cnt * K, c - cnt, key_type, R.st));
+        chunks[i] = R.stage;
+    }
+    MSORT_TRY(msort_sort_device(ctx, chunks.data(), c, nullptr));
+    for (int i = 0; i < n_gpus; ++i) {
+        Rank& R = ctx->r[i];
+        CUDA_TRY(cudaSetDevice(R.dev));
+        const uint64_t lo = std::min<uint64_t>(n, uint64_t(i) * c);
+        const uint64_t cnt = std::min<uint64_t>(n - lo, c);
+        if (cnt) CUDA_TRY(cudaMemcpyAsync(src + lo * K, R.stage, cnt * K, cudaMemcpyDefault, R.st));
+    }
+    for (int i = 0; i < n_gpus; ++i) {
+        CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
+        CUDA_TRY(cudaStreamSynchronize(ctx->r[i].st));
+    }
+    return MSORT_OK;
+}
+
+// --- dist mode (one process per GPU) -----------------------------------------
+
+struct DistHandle {
+    uint32_t magic;
+    int32_t rank;
+    uint64_t cap;
+    cudaIpcMemHandle_t b0, b1, flags;
+};
+static_assert(sizeof(DistHandle) <= MSORT_DIST_HANDLE_BYTES, "handle bytes");
+static const uint32_t kDistMagic = 0x4D534F52u;
+
+int msort_dist_create(msort_ctx** out, int rank, int world, int device, uint64_t max_keys_per_rank, int key_type) {
+    if (!out || !valid_g(world) || rank < 0 || rank >= world || !valid_kt(key_type))
+        return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad argument");
+    *out = nullptr;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        return set_error(MSORT_ERR_DEVICE, "no CUDA device");
+    }
+    if (device < 0 || device >= ndev) return set_error(MSORT_ERR_DEVICE, "device id out of range");
+    DeviceGuard guard;
+    auto ctx = std::make_unique<msort_ctx>();
+    ctx->g = world;
+    ctx->kt = key_type;
+    ctx->dist = true;
+    ctx->rank = rank;
+    ctx->nlocal = 1;
+    ctx->cap = (std::max<uint64_t>(max_keys_per_rank, 4) + 3) / 4 * 4;
+    if (ctx->cap >= (1ull << 32)) return set_error(MSORT_ERR_INVALID_ARGUMENT, "keys per GPU must be < 2^32");
+    ctx->r[0].dev = device;
+    int s = alloc_rank(ctx.get(), ctx->r[0], true, true);
+    if (s != MSORT_OK) {
+        free_rank(ctx->r[0]);
+        return s;
+    }
+    CUDA_TRY(cudaSetDevice(device));
+    CUDA_TRY(cudaMalloc(&ctx->my_flags, 256));
+    CUDA_TRY(cudaMemset(ctx->my_flags, 0, 256));
+    *out = ctx.release();
+    return MSORT_OK;
+}
+
+int msort_dist_export(msort_ctx* ctx, void* handle_out) {
+    if (!ctx || !ctx->dist || !handle_out) return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad argument");
+    DeviceGuard guard;
+    CUDA_TRY(cudaSetDevice(ctx->r[0].dev));
+    DistHandle h{};
+    h.magic = kDistMagic;
+    h.rank = ctx->rank;
+    h.cap = ctx->cap;
+    CUDA_TRY(cudaIpcGetMemHandle(&h.b0, ctx->r[0].buf[0]));
+    CUDA_TRY(cudaIpcGetMemHandle(&h.b1, ctx->r[0].buf[1]));
+    CUDA_TRY(cudaIpcGetMemHandle(&h.flags, ctx->my_flags));
+    std::memset(handle_out, 0, MSORT_DIST_HANDLE_BYTES);
+    std::memcpy(handle_out, &h, sizeof(h));
+    return MSORT_OK;
+}
+
+int msort_dist_import(msort_ctx* ctx, const void* all_handles) {
+    if (!ctx || !ctx->dist || !all_handles) return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad argument");
+    DeviceGuard guard;
+    CUDA_TRY(cudaSetDevice(ctx->r[0].dev));
+    const char* base = static_cast<const char*>(all_handles);
+    for (int q = 0; q < ctx->g; ++q) {
+        DistHandle h;
+        std::memcpy(&h, base + size_t(q) * MSORT_DIST_HANDLE_BYTES, sizeof(h));
+        if (h.magic != kDistMagic || h.rank != q || h.cap != ctx->cap)
+            return set_error(MSORT_ERR_INVALID_ARGUMENT, "handle array does not match (rank order / capacity)");
+        if (q == ctx->rank) {
+            ctx->peer_buf[q][0] = ctx->r[0].buf[0];
+            ctx->peer_buf[q][1] = ctx->r[0].buf[1];
+            ctx->peer_flags[q] = ctx->my_flags;
+            continue;
+        }
+        void* p = nullptr;
+        CUDA_TRY(cudaIpcOpenMemHandle(&p, h.b0, cudaIpcMemLazyEnablePeerAccess));
+        ctx->opened.push_back(p);
+        ctx->peer_buf[q][0] = p;
+        CUDA_TRY(cudaIpcOpenMemHandle(&p, h.b1, cudaIpcMemLazyEnablePeerAccess));
+        ctx->opened.push_back(p);
+        ctx->peer_buf[q][1] = p;
+        CUDA_TRY(cudaIpcOpenMemHandle(&p, h.flags, cudaIpcMemLazyEnablePeerAccess));
+        ctx->opened.push_back(p);
+        ctx->peer_flags[q] = static_cast<unsigned long long*>(p);
+    }
+    ctx->imported = true;
+    return MSORT_OK;
+}
+
+static int dist_barrier(msort_ctx* ctx) {
+    Rank& R = ctx->r[0];
+    BarrierArgs a{};
+    for (int q = 0; q < ctx->g; ++q) a.peer_flags[q] = ctx->peer_flags[q];
+    a.my_flags = ctx->my_flags;
+    a.rank = ctx->rank;
+    a.world = ctx->g;
+    a.epoch = ++ctx->epoch;
+    const char* env = std::getenv("MSORT_BARRIER_TIMEOUT_S");
+    const double tmo = env ? std::atof(env) : 60.0;
+    a.timeout_ns = (unsigned long long)(tmo * 1e9);
+    a.err = R.d_err;
+    CUDA_TRY(launch_barrier(a, R.st));
+    ctx->tm.kernel_launches += 1;
+    return MSORT_OK;
+}
+
+static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream, bool keep_timings);
+
+int msort_dist_sort(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream) {
+    return dist_sort_impl(ctx, d_chunk, c, stream, false);
+}
+
+int msort_dist_sort_host(msort_ctx* ctx, void* host_keys, uint64_t c) {
+    if (!ctx || !ctx->dist || !ctx->imported) return set_error(MSORT_ERR_INVALID_ARGUMENT, "dist ctx not imported");
+    if (c && !host_keys) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL keys");
+    MSORT_TRY(check_c(ctx, c));
+    DeviceGuard guard;
+    Rank& R = ctx->r[0];
+    CUDA_TRY(cudaSetDevice(R.dev));
+    reset_timings(ctx, c);
+    const size_t K = key_bytes(ctx->kt);
+    CUDA_TRY(cudaEventRecord(R.e_h2d0, R.st));
+    if (c) CUDA_TRY(cudaMemcpyAsync(R.stage, host_keys, c * K, cudaMemcpyHostToDevice, R.st));
+    CUDA_TRY(cudaEventRecord(R.e_h2d1, R.st));
+    MSORT_TRY(dist_sort_impl(ctx, R.stage, c, R.st, true));
+    CUDA_TRY(cudaEventRecord(R.e_d2h0, R.st));
+    if (c) CUDA_TRY(cudaMemcpyAsync(host_keys, R.stage, c * K, cudaMemcpyDeviceToHost, R.st));
+    CUDA_TRY(cudaEventRecord(R.e_d2h1, R.st));
+    CUDA_TRY(cudaEventSynchronize(R.e_d2h1));
+    ctx->tm.h2d_ms = elapsed(R.e_h2d0, R.e_h2d1);
+    ctx->tm.d2h_ms = elapsed(R.e_d2h0, R.e_d2h1);
+    ctx->tm.total_ms = elapsed(R.e_h2d0, R.e_d2h1);
+    return MSORT_OK;
+}
+
+static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream, bool keep_timings) {
+    if (!ctx || !ctx->dist || !ctx->imported) return set_error(MSORT_ERR_INVALID_ARGUMENT, "dist ctx not imported");
+    if (c && !d_chunk) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL chunk");
+    MSORT_TRY(check_c(ctx, c));
+    DeviceGuard guard;
+    const int g = ctx->g, me = ctx->rank;
+    Rank& R = ctx->r[0];
+    CUDA_TRY(cudaSetDevice(R.dev));
+    if (!keep_timings) reset_timings(ctx, c);
+    for (int s = 0; s < MSORT_MAX_STAGES; ++s)
+        for (auto& e : R.e_xch[s]) {
+            CUDA_TRY(cudaEventDestroy(e));
+            CUDA_TRY(cudaEventCreate(&e));
+        }
+    cudaStream_t ust = static_cast<cudaStream_t>(stream);
+    CUDA_TRY(cudaEventRecord(R.e_sync[MSORT_MAX_STAGES], ust));
+    CUDA_TRY(cudaStreamWaitEvent(R.st, R.e_sync[MSORT_MAX_STAGES], 0));
+    R.user = d_chunk;
+    CUDA_TRY(cudaEventRecord(R.e_begin, R.st));
+    if (c == 0) return MSORT_OK;
+    // S1-S3
+    MSORT_TRY(radix_begin(ctx, R, d_chunk, c));
+    if (ctx->skip_trivial) CUDA_TRY(cudaStreamSynchronize(R.st));
+    int cur[MSORT_MAX_GPUS];
+    if (g == 1) {
+        MSORT_TRY(radix_passes(ctx, R, d_chunk, d_chunk, R.buf[0], c));
+        for (int q = 0; q < g; ++q) cur[q] = -1;
+    } else {
+        MSORT_TRY(radix_passes(ctx, R, d_chunk, R.buf[1], R.buf[0], c));
+        for (int q = 0; q < g; ++q) cur[q] = 1;
+    }
+    CUDA_TRY(cudaEventRecord(R.e_sorted, R.st));
+    std::vector<int> labels;
+    stage_labels(g, labels);
+    const int S = int(labels.size());
+    ctx->tm.n_stages = S;
+    auto peer_ptr = [&](int q, int which) -> const void* {
+        return which < 0 ? (q == me ? d_chunk : nullptr) : ctx->peer_buf[q][which];
+    };
+    for (int s = 0; s < S; ++s) {
+        const int label = labels[s];
+        const bool last = s == S - 1;
+        MSORT_TRY(dist_barrier(ctx));
+        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[s][0], R.st));
+        GroupPtrs all{};
+        for (int q = 0; q < g; ++q) all.p[q] = peer_ptr(q, cur[q]);
+        const int ngroups = g / label;
+        CUDA_TRY(launch_pivots(all, ngroups, label, c, ctx->kt, R.d_pivot, R.st));
+        ctx->tm.kernel_launches += 1;
+        CUDA_TRY(cudaMemcpyAsync(R.h_pivot, R.d_pivot, ngroups * sizeof(uint64_t), cudaMemcpyDeviceToHost, R.st));
+        CUDA_TRY(cudaMemcpyAsync(R.h_err, R.d_err, sizeof(int), cudaMemcpyDeviceToHost, R.st));
+        CUDA_TRY(cudaStreamSynchronize(R.st));
+        if (*R.h_err) return set_error(MSORT_ERR_TIMEOUT, "device barrier timed out (a peer rank did not arrive)");
+        uint64_t piv[MSORT_MAX_GPUS / 2] = {};
+        for (int j = 0; j < ngroups; ++j) piv[j] = R.h_pivot[j];
+        Exchange ex;
+        plan_exchange(g, label, c, piv, ex);
+        ctx->tm.stage_label[s] = label;
+        uint64_t mx = 0, sum = 0;
+        for (int j = 0; j < ngroups; ++j) ctx->tm.stage_pivot[s][j] = piv[j];
+        for (int q = 0; q < g; ++q) {
+            mx = std::max(mx, ex.x[q]);
+            if (ex.side[q] == 0) sum += ex.x[q];
+        }
+        ctx->tm.stage_max_x[s] = mx;
+        ctx->tm.stage_keys_exchanged[s] = sum;
+        R.cur = cur[me];
+        int mine = cur[me];
+        const void* peer = ex.partner[me] >= 0 ? peer_ptr(ex.partner[me], cur[ex.partner[me]]) : nullptr;
+        MSORT_TRY(launch_exchange(ctx, R, s, last, c, ex.x[me], ex.side[me], peer_ptr(me, cur[me]), peer, mine));
+        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[s][1], R.st));
+        // replicate every rank's buffer rotation (all ranks see the same pivots)
+        for (int q = 0; q < g; ++q)
+            if (ex.x[q] != 0) cur[q] = last ? -1 : (cur[q] == 0 ? 1 : 0);
+        if (cur[me] != mine) return set_error(MSORT_ERR_INTERNAL, "buffer rotation diverged");
+    }
+    if (cur[me] != -1)
+        CUDA_TRY(cudaMemcpyAsync(d_chunk, ctx->peer_buf[me][cur[me]], c * key_bytes(ctx->kt), cudaMemcpyDeviceToDevice, R.st));
+    if (g > 1) MSORT_TRY(dist_barrier(ctx));  // peers finished reading our buffers before the next sort reuses them
+    CUDA_TRY(cudaEventRecord(R.e_end, R.st));
+    CUDA_TRY(cudaMemcpyAsync(R.h_err, R.d_err, sizeof(int), cudaMemcpyDeviceToHost, R.st));
+    CUDA_TRY(cudaStreamWaitEvent(ust, R.e_end, 0));
+    CUDA_TRY(cudaStreamSynchronize(R.st));
+    if (*R.h_err) return set_error(MSORT_ERR_TIMEOUT, "device barrier timed out (a peer rank did not arrive)");
+    collect_timings(ctx, 1);
+    collect_exchange_timings(ctx);
+    ctx->tm.total_ms = ctx->tm.sort_ms + ctx->tm.merge_ms;
+    return MSORT_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,265 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, bit-exact.
+
+Every row of SURVEY §8(a): S1+S2 histogram, S3 onesweep pass, S1-S3 radix sort,
+S4 pivot, S6 merge, S5+S6 fused exchange, S7 stage schedule (virtual ranks on
+one GPU), S0/S8 host round trip.  Sizes span several tiles and a ragged tail.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import msort_inputs as mi
+from oracle import codec, p2p, radix, sort
+
+pytestmark = pytest.mark.gpu
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+KT = {"u32": 0, "u64": 1, "f32": 2, "f64": 3}
+
+
+@pytest.fixture(scope="module")
+def ms():
+    if not torch.cuda.is_available():
+        pytest.fail("GPU tests need CUDA")
+    import paper_conf_sigmod_maltenbergeritr22_b200 as m
+    return m
+
+
+def dev_keys(a: np.ndarray) -> torch.Tensor:
+    return torch.from_numpy(a.view(np.uint8).copy()).cuda()
+
+
+def host_keys(t: torch.Tensor, kt: str) -> np.ndarray:
+    return t.cpu().numpy().view(mi.NP_DTYPE[kt])
+
+
+def bits(a, kt):
+    return codec.bits_of(a, kt)
+
+
+SIZES = [0, 1, 2, 3, 5, 100, 7679, 7680, 7681, 4608 * 3 + 17, 1 << 20, (1 << 20) + 13]
+
+
+@pytest.mark.parametrize("kt", ["u32", "u64", "f32", "f64"])
+@pytest.mark.parametrize("n", SIZES)
+def test_radix_sort_single_gpu(ms, kt, n):
+    a = mi.np_generate(n, kt, "uniform", seed=11)
+    d = dev_keys(a)
+    ms.msort_sort(ms.tensor_ptr(d), n, kt, 1)
+    torch.cuda.synchronize()
+    assert np.array_equal(bits(host_keys(d, kt), kt), bits(sort.oracle_sort(a, kt), kt))
+
+
+@pytest.mark.parametrize("dist", mi.DISTRIBUTIONS)
+def test_radix_sort_distributions(ms, dist):
+    n = 3 * (1 << 18) + 77
+    a = mi.np_generate(n, "u32", dist, seed=2)
+    d = dev_keys(a)
+    ms.msort_sort(ms.tensor_ptr(d), n, "u32", 1)
+    torch.cuda.synchronize()
+    assert np.array_equal(host_keys(d, "u32"), sort.oracle_sort(a, "u32"))
+
+
+def test_radix_sort_constant_and_special(ms):
+    # all-equal keys (every pass trivial) and the IEEE special-value table
+    for a, kt in [(np.full(50000, 7, np.uint32), "u32"), (np.full(9999, 0x7FC00000, np.uint32).view(np.float32), "f32")]:
+        d = dev_keys(a)
+        ms.msort_sort(ms.tensor_ptr(d), len(a), kt, 1)
+        torch.cuda.synchronize()
+        assert np.array_equal(bits(host_keys(d, kt), kt), bits(sort.oracle_sort(a, kt), kt))
+    with open(os.path.join(GOLD, "float_total_order_f32.json")) as f:
+        table = np.array([int(h, 16) for h in json.load(f)["ascending_bits_hex"]], dtype=np.uint32)
+    rng = np.random.default_rng(0)
+    a = table[rng.integers(0, len(table), 100000)].view(np.float32)
+    d = dev_keys(a)
+    ms.msort_sort(ms.tensor_ptr(d), len(a), "f32", 1)
+    torch.cuda.synchronize()
+    assert np.array_equal(host_keys(d, "f32").view(np.uint32), sort.oracle_sort(a, "f32").view(np.uint32))
+
+
+@pytest.mark.parametrize("kt", ["u32", "u64", "f32", "f64"])
+def test_step_histogram(ms, kt):
+    n = 123457
+    a = mi.np_generate(n, kt, "uniform", seed=3)
+    d = dev_keys(a)
+    P = radix.num_passes(kt)
+    h = torch.zeros(P * 256, dtype=torch.int32, device="cuda")
+    ms.msort_step_histogram(ms.tensor_ptr(d), n, kt, ms.tensor_ptr(h))
+    torch.cuda.synchronize()
+    got = h.cpu().numpy().view(np.uint32).reshape(P, 256)
+    assert np.array_equal(got.astype(np.uint64), radix.histograms(a, kt))
+
+
+@pytest.mark.parametrize("kt", ["u32", "u64", "f32"])
+def test_step_radix_pass(ms, kt):
+    n = 50001
+    a = mi.np_generate(n, kt, "uniform", seed=4)
+    P = radix.num_passes(kt)
+    hist = torch.from_numpy(radix.histograms(a, kt).astype(np.uint32).view(np.int32).reshape(-1).copy()).cuda()
+    ws_bytes = ms.msort_radix_workspace_bytes(n, kt)
+    ws = torch.empty(ws_bytes, dtype=torch.uint8, device="cuda")
+    codes = codec.encode(a, kt)
+    cur_dev = dev_keys(a)  # raw keys for pass 0
+    for p in range(P):
+        out = torch.empty_like(cur_dev)
+        flags = (ms.MSORT_PASS_ENCODE_IN if p == 0 else 0)
+        ms.msort_step_radix_pass(ms.tensor_ptr(cur_dev), ms.tensor_ptr(out), n, kt, p, ms.tensor_ptr(hist), flags,
+                                 ms.tensor_ptr(ws), ws_bytes)
+        torch.cuda.synchronize()
+        codes = radix.counting_pass(codes, p)
+        got = out.cpu().numpy().view(codec.UINT[kt])
+        assert np.array_equal(got, codes), f"pass {p}"
+        cur_dev = out
+
+
+def _chunks_to_dev(chunks, kt):
+    return [dev_keys(c) for c in chunks]
+
+
+@pytest.mark.parametrize("kt", ["u32", "u64", "f32"])
+@pytest.mark.parametrize("nchunks", [2, 4, 8])
+def test_step_pivot(ms, kt, nchunks):
+    rng = np.random.default_rng(nchunks)
+    for trial in range(12):
+        c = int(rng.integers(1, 3000))
+        dist = ["uniform", "sorted", "reverse"][trial % 3]
+        if kt == "u32":
+            data = mi.np_generate(c * nchunks, kt, "uniform", seed=trial)
+            if trial % 4 == 3:
+                data = (data % np.uint32(5)).astype(np.uint32)   # duplicate-heavy
+        else:
+            data = mi.np_generate(c * nchunks, kt, "uniform", seed=trial)
+        h = nchunks // 2
+        # A (left half) and B (right half) must each be sorted as concatenations
+        # (what the earlier merge stages guarantee)
+        A = sort.oracle_sort(data[: h * c], kt)
+        B = sort.oracle_sort(data[h * c:], kt)
+        if dist == "sorted":
+            s = sort.oracle_sort(data, kt)
+            A, B = s[: h * c], s[h * c:]
+        elif dist == "reverse":
+            s = sort.oracle_sort(data, kt)
+            A, B = s[h * c:], s[: h * c]
+        chunks = [A[i * c:(i + 1) * c] for i in range(h)] + [B[i * c:(i + 1) * c] for i in range(h)]
+        codes = [codec.encode(x, kt) for x in chunks]
+        expect = p2p.select_pivot(p2p.Concat(codes[:h]), p2p.Concat(codes[h:]))
+        devs = _chunks_to_dev(chunks, kt)
+        out = torch.zeros(1, dtype=torch.int64, device="cuda")
+        ms.msort_step_pivot([ms.tensor_ptr(t) for t in devs], c, kt, ms.tensor_ptr(out))
+        torch.cuda.synchronize()
+        assert int(out.item()) == expect
+
+
+def test_step_pivot_paper_figures(ms):
+    with open(os.path.join(GOLD, "fig8.json")) as f:
+        fx8 = json.load(f)
+    with open(os.path.join(GOLD, "fig9.json")) as f:
+        fx9 = json.load(f)
+    out = torch.zeros(1, dtype=torch.int64, device="cuda")
+    devs = [dev_keys(np.array(r, dtype=np.uint32)) for r in fx8["before"]]
+    ms.msort_step_pivot([ms.tensor_ptr(t) for t in devs], 4, "u32", ms.tensor_ptr(out))
+    torch.cuda.synchronize()
+    assert out.item() == fx8["pivot_p"]
+    devs = [dev_keys(np.array(r, dtype=np.uint32)) for r in fx9["after_stage1"]]
+    ms.msort_step_pivot([ms.tensor_ptr(t) for t in devs], 4, "u32", ms.tensor_ptr(out))
+    torch.cuda.synchronize()
+    assert out.item() == fx9["stage2_pivot_p"]
+
+
+@pytest.mark.parametrize("kt", ["u32", "u64", "f32", "f64"])
+def test_step_merge(ms, kt):
+    rng = np.random.default_rng(5)
+    for al, bl in [(0, 0), (0, 5), (7, 0), (1, 1), (3839, 1), (3840, 3840), (100000, 3), (54321, 65432)]:
+        a = sort.oracle_sort(mi.np_generate(al, kt, "uniform", seed=al + 1), kt)
+        b = sort.oracle_sort(mi.np_generate(bl, kt, "uniform", seed=bl + 2), kt)
+        if kt == "u32" and al and bl:
+            a = sort.oracle_sort((a % np.uint32(50)).astype(np.uint32), kt)   # ties across runs
+            b = sort.oracle_sort((b % np.uint32(50)).astype(np.uint32), kt)
+        da, db = dev_keys(a), dev_keys(b)
+        out = torch.zeros(max(1, (al + bl)) * mi.KEY_BYTES[kt], dtype=torch.uint8, device="cuda")
+        wsb = ms.msort_merge_workspace_bytes(al + bl, kt)
+        ws = torch.empty(wsb, dtype=torch.uint8, device="cuda")
+        ms.msort_step_merge(ms.tensor_ptr(da), al, ms.tensor_ptr(db), bl, ms.tensor_ptr(out), kt, ms.tensor_ptr(ws), wsb)
+        torch.cuda.synchronize()
+        got = host_keys(out, kt)[: al + bl]
+        expect = sort.oracle_sort(np.concatenate([a, b]), kt)
+        assert np.array_equal(bits(got, kt), bits(expect, kt)), (al, bl)
+
+
+def _virtual_sort(ms, a, kt, g, exchange=0):
+    """g virtual ranks on GPU 0, device-resident chunks of c keys."""
+    n = len(a)
+    c = n // g
+    ctx = ms.Context(g, n, kt, device_ids=[0] * g)
+    ctx.set_option(ms.MSORT_OPT_EXCHANGE, exchange)
+    chunks = [dev_keys(a[i * c:(i + 1) * c]) for i in range(g)]
+    ctx.sort_device([ms.tensor_ptr(t) for t in chunks], c)
+    torch.cuda.synchronize()
+    out = np.concatenate([host_keys(t, kt) for t in chunks])
+    tm = ctx.timings()
+    ctx.close()
+    return out, tm
+
+
+@pytest.mark.parametrize("g", [2, 4, 8])
+@pytest.mark.parametrize("dist", ["uniform", "sorted", "reverse", "nearly", "zipf"])
+def test_p2p_sort_virtual_ranks(ms, g, dist):
+    c = 3 * 7680 + 44
+    a = mi.np_generate(g * c, "u32", dist, seed=g)
+    out, tm = _virtual_sort(ms, a, "u32", g)
+    assert np.array_equal(out, sort.oracle_sort(a, "u32"))
+    # stage-level parity with the oracle's Alg.2 model: labels and every pivot
+    chunks = [np.sort(a[i * c:(i + 1) * c]) for i in range(g)]
+    stages = p2p.run_stages(chunks)
+    assert tm["stage_label"] == p2p.stage_labels(g)
+    for s, st in enumerate(stages):
+        assert tm["stage_pivot"][s][: len(st)] == [op.p for op in st]
+        assert tm["stage_max_x"][s] == max(max(op.xs) for op in st)
+
+
+@pytest.mark.parametrize("kt", ["u64", "f32", "f64"])
+def test_p2p_sort_virtual_key_types(ms, kt):
+    g, c = 4, 5000
+    a = mi.np_generate(g * c, kt, "uniform", seed=21)
+    out, _ = _virtual_sort(ms, a, kt, g)
+    assert np.array_equal(bits(out, kt), bits(sort.oracle_sort(a, kt), kt))
+
+
+@pytest.mark.parametrize("g", [2, 8])
+def test_p2p_sort_swap_mode(ms, g):
+    c = 20000
+    a = mi.np_generate(g * c, "u32", "uniform", seed=31)
+    out, tm = _virtual_sort(ms, a, "u32", g, exchange=1)
+    assert np.array_equal(out, sort.oracle_sort(a, "u32"))
+
+
+@pytest.mark.parametrize("g", [1, 2, 4, 8])
+@pytest.mark.parametrize("n", [2, 7, 1001, 65536 + 3])
+def test_sort_host_end_to_end(ms, g, n):
+    a = mi.np_generate(n, "u32", "uniform", seed=n)
+    h = torch.from_numpy(a.copy()).pin_memory()
+    ctx = ms.Context(g, n, "u32", device_ids=[0] * g)
+    ctx.sort_host(ms.tensor_ptr(h), n)
+    ctx.close()
+    assert np.array_equal(h.numpy(), sort.oracle_sort(a, "u32"))
+
+
+def test_msort_sort_host_pointer(ms):
+    n = 100003
+    a = mi.np_generate(n, "f32", "uniform", seed=9)
+    h = a.copy()
+    ms.msort_sort(h.ctypes.data, n, "f32", 1)
+    assert np.array_equal(h.view(np.uint32), sort.oracle_sort(a, "f32").view(np.uint32))
+
+
+def test_errors(ms):
+    with pytest.raises(ms.MsortError):
+        ms.msort_sort(0, 10, "u32", 1)
+    with pytest.raises(ms.MsortError):
+        ms.msort_sort(1234, 10, "u32", 3)
+    with pytest.raises(ms.MsortError):
+        ms.msort_sort(1234, 10, 9, 1)
+    ms.msort_sort(0, 0, "u32", 1)   # n = 0 is a no-op
