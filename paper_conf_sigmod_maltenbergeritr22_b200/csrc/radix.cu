@@ -5,13 +5,20 @@
 // the digit histogram is "calculated once" up front and the prefix sum is
 // "decoupled" (Thrust >= 1.11 / onesweep).  This file is a
 // from-scratch sm_100a onesweep:
-//   hist_kernel      one read of the chunk -> P digit histograms (S2)
+//   hist_kernel      one read of the chunk -> P digit histograms (S2); every
+//                    lane owns a private smem column per bin, so the smem
+//                    atomics of one warp instruction never collide on a bank
 //   scan_kernel      exclusive prefix per pass -> global digit bases (S2)
-//   onesweep_kernel  per tile: warp match-based stable ranking, block digit
-//                    counts, decoupled look-back across tiles for the global
-//                    digit offset, smem staging, coalesced scatter (S3)
+//   onesweep_kernel  persistent blocks; per tile: stable warp ranking (smem
+//                    atomicOr peer masks, or an 8-ballot match), block digit
+//                    counts, decoupled look-back across tiles with a 4-deep
+//                    window for the global digit offset, smem staging,
+//                    coalesced scatter (S3)
 // The float codec T (reading Q1) is applied on the first pass's load and T^-1
 // on the last pass's store (S1), so no separate codec pass touches HBM.
+#include <cstdlib>
+#include <type_traits>
+
 #include "common.cuh"
 #include "kernels.h"
 
@@ -19,28 +26,37 @@ namespace msort {
 
 namespace {
 
-constexpr int kHistThreads = 512;
-constexpr int kHistUnroll = 4;
-
 // ---------------------------------------------------------------------------
 // S2: digit histograms of T(key) for every pass, one read of the chunk.
-// Two sub-histograms per block (even/odd warps) halve same-bin smem atomic
-// collisions; each block flushes its counts with one global atomic per bin.
 // ---------------------------------------------------------------------------
+constexpr int kHistThreads = 1024;
+constexpr int kHistUnroll = 4;
+
+template <typename U>
+struct HistCfg {
+    static constexpr int P = sizeof(U);
+    static constexpr int REPL = sizeof(U) == 4 ? 32 : 16;  // private columns per bin
+    static constexpr size_t kSmem = size_t(P) * 256 * REPL * 4;  // 128 KB
+};
+
 template <typename U, bool FLOAT>
-__global__ void __launch_bounds__(kHistThreads) hist_kernel(const U* __restrict__ in, uint64_t n,
-                                                            uint32_t* __restrict__ hist) {
-    constexpr int P = sizeof(U);
+__global__ void __launch_bounds__(kHistThreads, 1) hist_kernel(const U* __restrict__ in, uint64_t n,
+                                                               uint32_t* __restrict__ hist) {
+    constexpr int P = HistCfg<U>::P;
+    constexpr int REPL = HistCfg<U>::REPL;
     constexpr int V = 16 / sizeof(U);  // keys per 16-byte vector
-    __shared__ uint32_t sh[2][P][kRadix];
-    for (int i = threadIdx.x; i < 2 * P * kRadix; i += blockDim.x) (&sh[0][0][0])[i] = 0;
+    extern __shared__ __align__(16) uint32_t sh[];  // [P][256][REPL]
+    {
+        uint4* s4 = reinterpret_cast<uint4*>(sh);
+        for (int i = threadIdx.x; i < P * 256 * REPL / 4; i += blockDim.x) s4[i] = make_uint4(0, 0, 0, 0);
+    }
     __syncthreads();
-    uint32_t(*my)[kRadix] = sh[(threadIdx.x >> 5) & 1];
+    const uint32_t col = threadIdx.x % REPL;
 
     auto count = [&](U k) {
         const U code = encode<U, FLOAT>(k);
 #pragma unroll
-        for (int p = 0; p < P; ++p) atomicAdd(&my[p][uint32_t(code >> (8 * p)) & 0xFF], 1u);
+        for (int p = 0; p < P; ++p) atomicAdd(&sh[((p << 8) + (uint32_t(code >> (8 * p)) & 0xFF)) * REPL + col], 1u);
     };
 
     const uintptr_t addr = reinterpret_cast<uintptr_t>(in);
@@ -73,9 +89,11 @@ __global__ void __launch_bounds__(kHistThreads) hist_kernel(const U* __restrict_
         for (uint64_t i = tail0 + threadIdx.x; i < n; i += blockDim.x) count(in[i]);
     }
     __syncthreads();
-    for (int i = threadIdx.x; i < P * kRadix; i += blockDim.x) {
-        const uint32_t s = (&sh[0][0][0])[i] + (&sh[1][0][0])[i];
-        if (s) atomicAdd(&hist[i], s);
+    for (int b = threadIdx.x; b < P * 256; b += blockDim.x) {
+        uint32_t s = 0;
+#pragma unroll 8
+        for (int j = 0; j < REPL; ++j) s += sh[b * REPL + ((j + b) % REPL)];  // rotated: no bank conflicts
+        if (s) atomicAdd(&hist[b], s);
     }
 }
 
@@ -107,226 +125,369 @@ __global__ void __launch_bounds__(kRadix) scan_kernel(const uint32_t* __restrict
 }
 
 // ---------------------------------------------------------------------------
-// S3: one onesweep pass.
+// S3: onesweep pass.
+//
+// B200 budget (measured, profiles/): at 80% of HBM a pass must move ~2.2
+// keys/cycle/SM, while shared memory serves 1 wavefront (128 B)/cycle/SM and
+// the integer ALU pipe 2 warp-instructions/cycle/SM; a random 4-byte smem
+// access by 32 lanes costs ~3.5 wavefronts (bank conflicts) and MATCH.ANY
+// ~60 ADU cycles.  The ranking therefore mixes two peer-mask methods per item
+// (compile-time pattern): an 8-ballot match (ALU only) and an smem atomicOr
+// mask (3 smem ops), so both pipes work in parallel.  Per-warp digit counts are
+// taken first ("early counts"), the tile aggregate is published before the
+// ranking, and the ranking's leader atomicAdd returns the final smem slot.
 // ---------------------------------------------------------------------------
 constexpr unsigned long long kFlagAgg = 1ull, kFlagIncl = 2ull;
+constexpr int kLookbackWindow = 4;
 
 __device__ __forceinline__ unsigned long long pack_status(unsigned long long flag, uint32_t tag, uint32_t count) {
     return (flag << 62) | (uint64_t(tag & 0x3FFFFFFFu) << 32) | count;
 }
 
-template <typename U>
-struct OnesweepCfg;
-template <>
-struct OnesweepCfg<uint32_t> {
-    static constexpr int kThreads = 384;
-    static constexpr int kItems = 20;
-};
-template <>
-struct OnesweepCfg<uint64_t> {
-    static constexpr int kThreads = 384;
-    static constexpr int kItems = 12;
+// Lanes of the warp whose 8-bit digit equals this lane's (8 ballots).
+__device__ __forceinline__ uint32_t ballot_match8(uint32_t d) {
+    uint32_t peers = 0xffffffffu;
+#pragma unroll
+    for (int b = 0; b < 8; ++b) {
+        asm("{\n\t.reg .pred p;\n\t.reg .b32 t, m;\n\t"
+            "and.b32 t, %1, %2;\n\t"
+            "setp.ne.u32 p, t, 0;\n\t"
+            "vote.sync.ballot.b32 m, p, 0xffffffff;\n\t"
+            "@!p not.b32 m, m;\n\t"
+            "and.b32 %0, %0, m;\n\t}"
+            : "+r"(peers)
+            : "r"(d), "r"(1u << b));
+    }
+    return peers;
+}
+
+// THREADS x ITEMS keys per tile; bit i of BALLOT_MASK: item i ranks with the
+// ballot match (else smem atomicOr); MINB blocks per SM for __launch_bounds__.
+template <int THREADS_, int ITEMS_, uint32_t BALLOT_MASK_, int MINB_>
+struct OsCfg {
+    static constexpr int kThreads = THREADS_;
+    static constexpr int kItems = ITEMS_;
+    static constexpr uint32_t kBallotMask = BALLOT_MASK_;
+    static constexpr int kMinBlocks = MINB_;
+    static constexpr int kWarps = THREADS_ / 32;
+    static constexpr uint32_t kTile = uint32_t(THREADS_) * ITEMS_;
+    static constexpr bool kAnyOr = (BALLOT_MASK_ & ((ITEMS_ >= 32 ? 0u : (1u << ITEMS_)) - 1u)) !=
+                                   ((ITEMS_ >= 32 ? 0u : (1u << ITEMS_)) - 1u);
+    template <typename U>
+    static constexpr size_t smem_bytes() {
+        return 2 * size_t(kTile) * sizeof(U) + size_t(kWarps) * kRadix * 4 * (kAnyOr ? 2 : 1);
+    }
 };
 
-template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT>
-__global__ void __launch_bounds__(OnesweepCfg<U>::kThreads, 2)
+template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg>
+__global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     onesweep_kernel(const U* __restrict__ in, U* __restrict__ out, uint32_t n, uint32_t shift,
                     const uint32_t* __restrict__ base, unsigned long long* __restrict__ status,
                     uint32_t* __restrict__ tile_counter, uint32_t tag) {
-    constexpr int THREADS = OnesweepCfg<U>::kThreads;
-    constexpr int ITEMS = OnesweepCfg<U>::kItems;
-    constexpr int WARPS = THREADS / 32;
-    constexpr uint32_t TILE = THREADS * ITEMS;
+    constexpr int THREADS = Cfg::kThreads;
+    constexpr int ITEMS = Cfg::kItems;
+    constexpr int WARPS = Cfg::kWarps;
+    constexpr uint32_t TILE = Cfg::kTile;
     static_assert(THREADS >= kRadix, "one thread per digit in the look-back");
+    static_assert((TILE * sizeof(U)) % 16 == 0, "bulk copies move whole 16-byte units");
 
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    U* s_keys = reinterpret_cast<U*>(smem_raw);
-    __shared__ uint32_t s_wcnt[WARPS][kRadix];  // per-warp digit counts, then per-warp exclusive offsets
-    __shared__ uint32_t s_total[kRadix];
-    __shared__ uint32_t s_dstart[kRadix];
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    U* s_in = reinterpret_cast<U*>(smem_raw);                             // TMA-prefetched input tile
+    U* s_keys = s_in + TILE;                                              // digit-ordered staging
+    uint32_t(*s_cnt)[kRadix] = reinterpret_cast<uint32_t(*)[kRadix]>(s_keys + TILE);
+    uint32_t(*s_match)[kRadix] = s_cnt + WARPS;  // only touched by atomicOr-ranked items
     __shared__ uint32_t s_delta[kRadix];
     __shared__ uint32_t s_wsum[kRadix / 32];
-    __shared__ uint32_t s_tile;
+    __shared__ uint32_t s_next;
+    __shared__ __align__(8) uint64_t s_bar;
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    // Tile ids in launch-independent arrival order: every lower tile has
-    // already started, so the look-back below always makes progress.
-    if (tid == 0) s_tile = atomicAdd(tile_counter, 1u);
-    for (int i = tid; i < WARPS * kRadix; i += THREADS) (&s_wcnt[0][0])[i] = 0;
-    __syncthreads();
-    const uint32_t tile = s_tile;
-    const uint64_t tile_base = uint64_t(tile) * TILE;
-    const bool full = tile_base + TILE <= n;
-
-    // --- load (warp-striped: warp w owns keys [w*32*ITEMS, (w+1)*32*ITEMS) of the tile)
-    U keys[ITEMS];
-    const uint64_t first = tile_base + uint64_t(warp) * 32 * ITEMS + lane;
-    const U* src = in + first;
-    if (full) {
-#pragma unroll
-        for (int i = 0; i < ITEMS; ++i) keys[i] = __ldcs(src + i * 32);
-#pragma unroll
-        for (int i = 0; i < ITEMS; ++i)
-            if (ENC_IN) keys[i] = encode<U, FLOAT>(keys[i]);
-    } else {
-        // out-of-range slots get the largest code: they rank after every real
-        // key of digit 255 and are never stored (see scatter bound)
-#pragma unroll
-        for (int i = 0; i < ITEMS; ++i) {
-            const bool ok = first + uint64_t(i) * 32 < n;
-            U k = ok ? src[i * 32] : U(0);
-            if (ENC_IN) k = encode<U, FLOAT>(k);
-            keys[i] = ok ? k : ~U(0);
-        }
-    }
-
-    // --- stable warp-level ranking: peers with the same digit via match.any;
-    // the lowest peer bumps the warp's digit counter for the whole group.
-    uint32_t rk[ITEMS];
+    const uint32_t ntiles = (n + TILE - 1) / TILE;
     const uint32_t lt = lanemask_lt();
-#pragma unroll
-    for (int i = 0; i < ITEMS; ++i) {
-        const uint32_t d = uint32_t(keys[i] >> shift) & 0xFF;
-        const uint32_t peers = __match_any_sync(0xffffffffu, d);
-        const uint32_t below = __popc(peers & lt);
-        const int leader = __ffs(peers) - 1;
-        uint32_t old = 0;
-        if (below == 0) old = atomicAdd(&s_wcnt[warp][d], uint32_t(__popc(peers)));
-        old = __shfl_sync(0xffffffffu, old, leader);
-        rk[i] = (old + below) | (d << 16);
+    // the TMA path needs a 16-byte aligned source; full tiles only
+    const bool aligned = (reinterpret_cast<uintptr_t>(in) & 15) == 0;
+    auto tma_ok = [&](uint32_t t) { return aligned && uint64_t(t + 1) * TILE <= n; };
+
+    if (Cfg::kAnyOr) {
+        for (int i = tid; i < WARPS * kRadix; i += THREADS) (&s_match[0][0])[i] = 0;
+    }
+    if (tid == 0) {
+        mbar_init(&s_bar, 1);
+        // Tile ids in arrival order: every lower tile is already held by a
+        // running block, so the look-back below always makes progress.
+        const uint32_t t0 = atomicAdd(tile_counter, 1u);
+        s_next = t0;
+        if (t0 < ntiles && tma_ok(t0)) tma_load_1d(s_in, in + uint64_t(t0) * TILE, TILE * sizeof(U), &s_bar);
     }
     __syncthreads();
+    uint32_t parity = 0;
 
-    // --- block digit totals, per-warp exclusive offsets; publish aggregates
-    if (tid < kRadix) {
-        const int d = tid;
-        uint32_t sum = 0;
-#pragma unroll
-        for (int w = 0; w < WARPS; ++w) {
-            const uint32_t c = s_wcnt[w][d];
-            s_wcnt[w][d] = sum;
-            sum += c;
-        }
-        s_total[d] = sum;
-        st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(tile == 0 ? kFlagIncl : kFlagAgg, tag, sum));
-        // block exclusive scan of totals over digits -> local digit starts
-        uint32_t x = sum;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-            if (lane >= o) x += y;
-        }
-        if (lane == 31) s_wsum[warp] = x;
-        s_dstart[d] = x - sum;  // warp-local exclusive; warp prefix added below
-    }
-    __syncthreads();
-    if (tid < kRadix) {
-        uint32_t pre = 0;
-        for (int w = 0; w < (tid >> 5); ++w) pre += s_wsum[w];
-        s_dstart[tid] += pre;
-    }
-    __syncthreads();
+    for (;;) {
+        const uint32_t tile = s_next;
+        if (tile >= ntiles) break;
+        const uint64_t tile_base = uint64_t(tile) * TILE;
+        const bool full = tile_base + TILE <= n;
 
-    // --- stage keys in smem in tile-local digit order
+        // --- keys -> registers (warp-striped: warp w owns keys [w*32*ITEMS, (w+1)*32*ITEMS))
+        U keys[ITEMS];
+        const uint32_t wofs = uint32_t(warp) * 32 * ITEMS + lane;
+        if (tma_ok(tile)) {
+            mbar_wait(&s_bar, parity);
+            parity ^= 1;
 #pragma unroll
-    for (int i = 0; i < ITEMS; ++i) {
-        const uint32_t d = rk[i] >> 16;
-        const uint32_t pos = s_dstart[d] + s_wcnt[warp][d] + (rk[i] & 0xFFFF);
-        s_keys[pos] = keys[i];
-    }
-
-    // --- decoupled look-back: exclusive count of digit d over all earlier tiles
-    if (tid < kRadix) {
-        const int d = tid;
-        uint32_t excl = 0;
-        if (tile > 0) {
-            int64_t t = int64_t(tile) - 1;
-            while (true) {
-                const unsigned long long w = ld_relaxed_gpu(&status[uint64_t(t) * kRadix + d]);
-                const unsigned long long flag = w >> 62;
-                const uint32_t wtag = uint32_t(w >> 32) & 0x3FFFFFFFu;
-                if (flag == 0 || wtag != (tag & 0x3FFFFFFFu)) continue;  // predecessor not published yet
-                excl += uint32_t(w);
-                if (flag == kFlagIncl) break;
-                --t;
+            for (int i = 0; i < ITEMS; ++i) keys[i] = s_in[wofs + i * 32];
+#pragma unroll
+            for (int i = 0; i < ITEMS; ++i)
+                if (ENC_IN) keys[i] = encode<U, FLOAT>(keys[i]);
+        } else {
+            // out-of-range slots get the largest code: they rank after every real
+            // key of digit 255 and are never stored (see the scatter bound)
+            const U* src = in + tile_base + wofs;
+#pragma unroll
+            for (int i = 0; i < ITEMS; ++i) {
+                const bool ok = tile_base + wofs + uint64_t(i) * 32 < n;
+                U k = ok ? src[i * 32] : U(0);
+                if (ENC_IN) k = encode<U, FLOAT>(k);
+                keys[i] = ok ? k : ~U(0);
             }
-            st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(kFlagIncl, tag, excl + s_total[d]));
         }
-        s_delta[d] = base[d] + excl - s_dstart[d];
-    }
-    __syncthreads();
+        {
+            uint4* z = reinterpret_cast<uint4*>(&s_cnt[0][0]);
+            for (int i = tid; i < WARPS * kRadix / 4; i += THREADS) z[i] = make_uint4(0, 0, 0, 0);
+        }
+        __syncthreads();  // s_in fully consumed, s_cnt zeroed
 
-    // --- scatter: consecutive smem slots of one digit go to consecutive output slots
-    if (full) {
+        // --- prefetch the next tile into s_in while this one is ranked and scattered
+        if (tid == 0) {
+            const uint32_t nx = atomicAdd(tile_counter, 1u);
+            s_next = nx;
+            if (nx < ntiles && tma_ok(nx)) tma_load_1d(s_in, in + uint64_t(nx) * TILE, TILE * sizeof(U), &s_bar);
+        }
+
+        // --- early counts: per-warp digit histogram (fire-and-forget smem adds)
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) atomicAdd(&s_cnt[warp][uint32_t(keys[i] >> shift) & 0xFF], 1u);
+        __syncthreads();
+
+        // --- tile totals -> publish aggregate; per-(warp, digit) smem slot bases
+        uint32_t my_total = 0, my_start = 0;
+        if (tid < kRadix) {
+            const int d = tid;
+            uint32_t sum = 0;
+#pragma unroll
+            for (int w = 0; w < WARPS; ++w) sum += s_cnt[w][d];
+            my_total = sum;
+            st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(tile == 0 ? kFlagIncl : kFlagAgg, tag, sum));
+            uint32_t x = sum;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+                if (lane >= o) x += y;
+            }
+            if (lane == 31) s_wsum[warp] = x;
+            my_start = x - sum;  // warp-local exclusive
+        }
+        __syncthreads();
+        if (tid < kRadix) {
+            uint32_t pre = 0;
+            for (int w = 0; w < (tid >> 5); ++w) pre += s_wsum[w];
+            my_start += pre;
+            uint32_t run = my_start;
+#pragma unroll
+            for (int w = 0; w < WARPS; ++w) {
+                const uint32_t c = s_cnt[w][tid];
+                s_cnt[w][tid] = run;
+                run += c;
+            }
+        }
+        __syncthreads();
+
+        // --- stable warp ranking straight into the smem slot (tile-local digit order)
 #pragma unroll
         for (int i = 0; i < ITEMS; ++i) {
-            const uint32_t j = tid + i * THREADS;
-            const U k = s_keys[j];
-            const uint32_t dst = s_delta[uint32_t(k >> shift) & 0xFF] + j;
-            __stcs(out + dst, DEC_OUT ? decode<U, FLOAT>(k) : k);
+            const uint32_t d = uint32_t(keys[i] >> shift) & 0xFF;
+            uint32_t peers;
+            if ((Cfg::kBallotMask >> i) & 1u) {
+                peers = ballot_match8(d);
+            } else {
+                atomicOr(&s_match[warp][d], 1u << lane);
+                __syncwarp();
+                peers = *reinterpret_cast<volatile uint32_t*>(&s_match[warp][d]);
+            }
+            const int leader = 31 - __clz(peers);
+            uint32_t slot = 0;
+            if (lane == leader) slot = atomicAdd(&s_cnt[warp][d], uint32_t(__popc(peers)));
+            slot = __shfl_sync(0xffffffffu, slot, leader) + __popc(peers & lt);
+            if (!((Cfg::kBallotMask >> i) & 1u)) {
+                if (lane == leader) s_match[warp][d] = 0;
+                __syncwarp();
+            }
+            s_keys[slot] = keys[i];
         }
-    } else {
-        const uint32_t valid = uint32_t(n - tile_base);
-        for (uint32_t j = tid; j < valid; j += THREADS) {
-            const U k = s_keys[j];
-            const uint32_t dst = s_delta[uint32_t(k >> shift) & 0xFF] + j;
-            out[dst] = DEC_OUT ? decode<U, FLOAT>(k) : k;
+
+        // --- decoupled look-back: exclusive count of digit d over all earlier tiles.
+        // Deferred until after the ranking so predecessors had time to publish;
+        // a 4-wide first probe, then 16-wide windows over runs of aggregates.
+        if (tid < kRadix) {
+            const int d = tid;
+            uint32_t excl = 0;
+            if (tile > 0) {
+                const uint32_t tg = tag & 0x3FFFFFFFu;
+                int64_t t = int64_t(tile) - 1;
+                const unsigned long long* p = status + uint64_t(t) * kRadix + d;
+                bool done = false;
+                auto probe = [&](auto W) {
+                    constexpr int kW = decltype(W)::value;
+                    unsigned long long w[kW];
+#pragma unroll
+                    for (int k = 0; k < kW; ++k) w[k] = (t - k >= 0) ? ld_relaxed_gpu(p - k * kRadix) : 0ull;
+                    int used = 0;
+#pragma unroll
+                    for (int k = 0; k < kW; ++k) {
+                        if (done || used < k) continue;
+                        const unsigned long long flag = w[k] >> 62;
+                        if (flag == 0 || (uint32_t(w[k] >> 32) & 0x3FFFFFFFu) != tg) continue;  // not published yet
+                        excl += uint32_t(w[k]);
+                        used = k + 1;
+                        if (flag == kFlagIncl) done = true;
+                    }
+                    t -= used;
+                    p -= used * kRadix;
+                    return used;
+                };
+                int used = probe(std::integral_constant<int, 4>{});
+                while (!done) {
+                    if (used == 0) __nanosleep(64);
+                    used = probe(std::integral_constant<int, 16>{});
+                }
+                st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(kFlagIncl, tag, excl + my_total));
+            }
+            s_delta[d] = base[d] + excl - my_start;
         }
+        __syncthreads();
+
+        // --- scatter: consecutive smem slots of one digit go to consecutive output slots
+        if (full) {
+#pragma unroll
+            for (int i = 0; i < ITEMS; ++i) {
+                const uint32_t j = tid + i * THREADS;
+                const U k = s_keys[j];
+                const uint32_t dst = s_delta[uint32_t(k >> shift) & 0xFF] + j;
+                __stcs(out + dst, DEC_OUT ? decode<U, FLOAT>(k) : k);
+            }
+        } else {
+            const uint32_t valid = uint32_t(n - tile_base);
+            for (uint32_t j = tid; j < valid; j += THREADS) {
+                const U k = s_keys[j];
+                const uint32_t dst = s_delta[uint32_t(k >> shift) & 0xFF] + j;
+                out[dst] = DEC_OUT ? decode<U, FLOAT>(k) : k;
+            }
+        }
+        __syncthreads();
     }
+    // a prefetch issued for an out-of-range id never happens (guarded above), so
+    // no bulk copy is in flight when the block exits
+}
+// Tile configurations (selectable with MSORT_OS_CFG for tuning; 0 = default).
+using Cfg32_0 = OsCfg<384, 20, 0x55555u, 2>;   // alternate ballot / atomicOr (84 KB smem)
+using Cfg32_1 = OsCfg<256, 20, 0xFFFFFu, 4>;   // all ballot, 4 blocks of 256 (48 KB)
+using Cfg32_2 = OsCfg<256, 20, 0x55555u, 3>;   // alternate, 3 blocks of 256 (56 KB)
+using Cfg32_3 = OsCfg<512, 16, 0x5555u, 2>;    // alternate, 2 blocks of 512 (96 KB)
+using Cfg64_0 = OsCfg<384, 12, 0x555u, 2>;
+using Cfg64_1 = OsCfg<256, 12, 0xFFFu, 3>;
+using Cfg64_2 = OsCfg<256, 12, 0x555u, 3>;
+using Cfg64_3 = OsCfg<512, 8, 0x55u, 2>;
+
+constexpr uint32_t kMinTile32 = 256 * 20;
+constexpr uint32_t kMinTile64 = 256 * 12;  // smallest u64 tile above
+
+int env_cfg() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = std::getenv("MSORT_OS_CFG");
+        v = e ? std::atoi(e) : 0;
+        if (v < 0 || v > 3) v = 0;
+    }
+    return v;
+}
+
+int sm_count() {
+    int dev = 0, count = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&count, cudaDevAttrMultiProcessorCount, dev);
+    return count > 0 ? count : 148;
+}
+
+template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg>
+cudaError_t launch_onesweep_c(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
+                              const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
+    const size_t smem = Cfg::template smem_bytes<U>();
+    auto kern = onesweep_kernel<U, FLOAT, ENC_IN, DEC_OUT, Cfg>;
+    // per-device attribute: set on every launch (cheap, and correct when one
+    // process drives several GPUs)
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    if (e != cudaSuccess) return e;
+    int per_sm = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, Cfg::kThreads, smem);
+    if (e != cudaSuccess) return e;
+    if (per_sm < 1) per_sm = 1;
+    const uint64_t tiles = (n + Cfg::kTile - 1) / Cfg::kTile;
+    uint64_t grid = uint64_t(per_sm) * sm_count();
+    if (grid > tiles) grid = tiles;
+    kern<<<unsigned(grid), Cfg::kThreads, smem, st>>>(reinterpret_cast<const U*>(in), reinterpret_cast<U*>(out),
+                                                     uint32_t(n), uint32_t(8 * pass), base_row, ws.status,
+                                                     ws.counters + pass, tag);
+    return cudaGetLastError();
 }
 
 template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT>
 cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
                               const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
-    using Cfg = OnesweepCfg<U>;
-    constexpr uint32_t TILE = Cfg::kThreads * Cfg::kItems;
-    const size_t smem = size_t(TILE) * sizeof(U);
-    auto kern = onesweep_kernel<U, FLOAT, ENC_IN, DEC_OUT>;
-    // per-device attribute: set on every launch (cheap, and correct when one
-    // process drives several GPUs)
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-    if (e != cudaSuccess) return e;
-    const uint64_t tiles = (n + TILE - 1) / TILE;
-    kern<<<unsigned(tiles), Cfg::kThreads, smem, st>>>(reinterpret_cast<const U*>(in), reinterpret_cast<U*>(out),
-                                                      uint32_t(n), uint32_t(8 * pass), base_row, ws.status,
-                                                      ws.counters + pass, tag);
-    return cudaGetLastError();
-}
-
-template <typename U, bool FLOAT>
-cudaError_t launch_onesweep_f(const void* in, void* out, uint64_t n, int pass, int flags, const RadixWs& ws,
-                              const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
-    const bool enc = flags & 1, dec = flags & 2;
-    if (!FLOAT || (!enc && !dec)) return launch_onesweep_t<U, FLOAT, false, false>(in, out, n, pass, ws, base_row, tag, st);
-    if (enc && dec) return launch_onesweep_t<U, FLOAT, true, true>(in, out, n, pass, ws, base_row, tag, st);
-    if (enc) return launch_onesweep_t<U, FLOAT, true, false>(in, out, n, pass, ws, base_row, tag, st);
-    return launch_onesweep_t<U, FLOAT, false, true>(in, out, n, pass, ws, base_row, tag, st);
-}
-
-int sm_count() {
-    static int count = 0;
-    if (!count) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&count, cudaDevAttrMultiProcessorCount, dev);
-        if (count <= 0) count = 148;
+    const int c = env_cfg();
+    if constexpr (sizeof(U) == 4) {
+        switch (c) {
+            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_1>(in, out, n, pass, ws, base_row, tag, st);
+            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_2>(in, out, n, pass, ws, base_row, tag, st);
+            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_3>(in, out, n, pass, ws, base_row, tag, st);
+            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_0>(in, out, n, pass, ws, base_row, tag, st);
+        }
+    } else {
+        switch (c) {
+            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_1>(in, out, n, pass, ws, base_row, tag, st);
+            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_2>(in, out, n, pass, ws, base_row, tag, st);
+            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_3>(in, out, n, pass, ws, base_row, tag, st);
+            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0>(in, out, n, pass, ws, base_row, tag, st);
+        }
     }
-    return count;
+}
+
+template <typename U>
+cudaError_t launch_onesweep_int(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
+                                const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
+    return launch_onesweep_t<U, false, false, false>(in, out, n, pass, ws, base_row, tag, st);
+}
+
+template <typename U>
+cudaError_t launch_onesweep_float(const void* in, void* out, uint64_t n, int pass, int flags, const RadixWs& ws,
+                                  const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
+    const bool enc = flags & 1, dec = flags & 2;
+    if (enc && dec) return launch_onesweep_t<U, true, true, true>(in, out, n, pass, ws, base_row, tag, st);
+    if (enc) return launch_onesweep_t<U, true, true, false>(in, out, n, pass, ws, base_row, tag, st);
+    if (dec) return launch_onesweep_t<U, true, false, true>(in, out, n, pass, ws, base_row, tag, st);
+    return launch_onesweep_t<U, true, false, false>(in, out, n, pass, ws, base_row, tag, st);
 }
 
 }  // namespace
 
-uint32_t radix_tile_keys(int kt) {
-    return key_bytes(kt) == 4 ? OnesweepCfg<uint32_t>::kThreads * OnesweepCfg<uint32_t>::kItems
-                              : OnesweepCfg<uint64_t>::kThreads * OnesweepCfg<uint64_t>::kItems;
-}
+uint32_t radix_tile_keys(int kt) { return key_bytes(kt) == 4 ? kMinTile32 : kMinTile64; }
 
 static size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
+static size_t head_bytes() { return align_up(8 * 4 + 8 * 256 * 4 * 2 + 8 * 4, 256); }
+
 size_t radix_ws_bytes(uint64_t n, int kt) {
     const uint64_t tiles = (n + radix_tile_keys(kt) - 1) / radix_tile_keys(kt);
-    const size_t head = align_up(8 * 4 + 8 * 256 * 4 * 2 + 8 * 4, 256);
-    return head + align_up(size_t(tiles) * kRadix * 8, 256) + 256;
+    return head_bytes() + align_up(size_t(tiles) * kRadix * 8, 256) + 256;
 }
 
 RadixWs radix_ws_layout(void* ws, uint64_t n, int kt) {
@@ -336,29 +497,37 @@ RadixWs radix_ws_layout(void* ws, uint64_t n, int kt) {
     w.hist = w.counters + 8;
     w.base = w.hist + 8 * 256;
     w.trivial = w.base + 8 * 256;
-    w.head_bytes = align_up(8 * 4 + 8 * 256 * 4 * 2 + 8 * 4, 256);
+    w.head_bytes = head_bytes();
     w.status = reinterpret_cast<unsigned long long*>(p + w.head_bytes);
     w.tiles = (n + radix_tile_keys(kt) - 1) / radix_tile_keys(kt);
     return w;
+}
+
+template <typename U, bool FLOAT>
+static cudaError_t launch_hist_t(const void* keys, uint64_t n, uint32_t* hist, cudaStream_t st) {
+    auto kern = hist_kernel<U, FLOAT>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(HistCfg<U>::kSmem));
+    if (e != cudaSuccess) return e;
+    const uint64_t vec = n / (16 / sizeof(U)) + 1;
+    uint64_t blocks = (vec + uint64_t(kHistThreads) * kHistUnroll - 1) / (uint64_t(kHistThreads) * kHistUnroll);
+    const uint64_t cap = uint64_t(sm_count());
+    if (blocks > cap) blocks = cap;
+    if (blocks == 0) blocks = 1;
+    kern<<<unsigned(blocks), kHistThreads, HistCfg<U>::kSmem, st>>>(reinterpret_cast<const U*>(keys), n, hist);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_histogram(const void* keys, uint64_t n, int kt, uint32_t* hist, cudaStream_t st) {
     const int P = num_passes(kt);
     cudaError_t e = cudaMemsetAsync(hist, 0, size_t(P) * kRadix * 4, st);
     if (e != cudaSuccess || n == 0) return e;
-    const uint64_t vec = n / (16 / key_bytes(kt)) + 1;
-    uint64_t blocks = (vec + kHistThreads * kHistUnroll - 1) / (kHistThreads * kHistUnroll);
-    const uint64_t cap = uint64_t(sm_count()) * 4;
-    if (blocks > cap) blocks = cap;
-    if (blocks == 0) blocks = 1;
     switch (kt) {
-        case 0: hist_kernel<uint32_t, false><<<unsigned(blocks), kHistThreads, 0, st>>>((const uint32_t*)keys, n, hist); break;
-        case 1: hist_kernel<uint64_t, false><<<unsigned(blocks), kHistThreads, 0, st>>>((const uint64_t*)keys, n, hist); break;
-        case 2: hist_kernel<uint32_t, true><<<unsigned(blocks), kHistThreads, 0, st>>>((const uint32_t*)keys, n, hist); break;
-        case 3: hist_kernel<uint64_t, true><<<unsigned(blocks), kHistThreads, 0, st>>>((const uint64_t*)keys, n, hist); break;
+        case 0: return launch_hist_t<uint32_t, false>(keys, n, hist, st);
+        case 1: return launch_hist_t<uint64_t, false>(keys, n, hist, st);
+        case 2: return launch_hist_t<uint32_t, true>(keys, n, hist, st);
+        case 3: return launch_hist_t<uint64_t, true>(keys, n, hist, st);
         default: return cudaErrorInvalidValue;
     }
-    return cudaGetLastError();
 }
 
 cudaError_t launch_scan(const uint32_t* hist, uint32_t* base, uint32_t* trivial, uint64_t n, int kt, cudaStream_t st) {
@@ -378,10 +547,10 @@ cudaError_t launch_onesweep(const void* in, void* out, uint64_t n, int kt, int p
     if (n == 0) return cudaSuccess;
     const uint32_t tag = uint32_t(pass) + 1;  // status words of other passes are ignored
     switch (kt) {
-        case 0: return launch_onesweep_f<uint32_t, false>(in, out, n, pass, flags, ws, base_row, tag, st);
-        case 1: return launch_onesweep_f<uint64_t, false>(in, out, n, pass, flags, ws, base_row, tag, st);
-        case 2: return launch_onesweep_f<uint32_t, true>(in, out, n, pass, flags, ws, base_row, tag, st);
-        case 3: return launch_onesweep_f<uint64_t, true>(in, out, n, pass, flags, ws, base_row, tag, st);
+        case 0: return launch_onesweep_int<uint32_t>(in, out, n, pass, ws, base_row, tag, st);
+        case 1: return launch_onesweep_int<uint64_t>(in, out, n, pass, ws, base_row, tag, st);
+        case 2: return launch_onesweep_float<uint32_t>(in, out, n, pass, flags, ws, base_row, tag, st);
+        case 3: return launch_onesweep_float<uint64_t>(in, out, n, pass, flags, ws, base_row, tag, st);
         default: return cudaErrorInvalidValue;
     }
 }
