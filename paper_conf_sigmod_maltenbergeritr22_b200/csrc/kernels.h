@@ -19,7 +19,8 @@ struct RadixWs {
     uint32_t* trivial;            // [8] 1 if the pass's digit is constant over all keys
     unsigned long long* status;   // [tiles][256] decoupled-lookback words
     uint64_t tiles;
-    size_t head_bytes;            // bytes of counters..trivial (zeroed per sort)
+    size_t head_bytes;            // bytes of counters..trivial
+    size_t zero_bytes;            // head + status words: zeroed once per sort
 };
 uint32_t radix_tile_keys(int kt);
 size_t radix_ws_bytes(uint64_t n, int kt);

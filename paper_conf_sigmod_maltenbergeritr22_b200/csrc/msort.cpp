@@ -558,7 +558,7 @@ int msort_step_radix_pass(const void* d_in, void* d_out, uint64_t n, int key_typ
     if (ws_bytes < radix_ws_bytes(n, key_type) || !d_ws) return set_error(MSORT_ERR_INVALID_ARGUMENT, "workspace too small");
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     RadixWs ws = radix_ws_layout(d_ws, n, key_type);
-    CUDA_TRY(cudaMemsetAsync(ws.counters, 0, ws.head_bytes + size_t(ws.tiles) * 256 * 8, st));
+    CUDA_TRY(cudaMemsetAsync(ws.counters, 0, ws.zero_bytes, st));
     CUDA_TRY(launch_scan(d_hist, ws.base, ws.trivial, n, key_type, st));
     CUDA_TRY(launch_onesweep(d_in, d_out, n, key_type, pass, flags & 3, ws, ws.base + pass * 256, st));
     return MSORT_OK;

@@ -163,8 +163,9 @@ __device__ __forceinline__ uint32_t ballot_match8(uint32_t d) {
 
 // THREADS x ITEMS keys per tile; bit i of BALLOT_MASK: item i ranks with the
 // ballot match (else smem atomicOr); MINB blocks per SM for __launch_bounds__.
-template <int THREADS_, int ITEMS_, uint32_t BALLOT_MASK_, int MINB_>
+template <int THREADS_, int ITEMS_, uint32_t BALLOT_MASK_, int MINB_, bool TMA_>
 struct OsCfg {
+    static constexpr bool kTma = TMA_;  // bulk-copy (TMA) the next tile into smem during the scatter
     static constexpr int kThreads = THREADS_;
     static constexpr int kItems = ITEMS_;
     static constexpr uint32_t kBallotMask = BALLOT_MASK_;
@@ -175,7 +176,7 @@ struct OsCfg {
                                    ((ITEMS_ >= 32 ? 0u : (1u << ITEMS_)) - 1u);
     template <typename U>
     static constexpr size_t smem_bytes() {
-        return 2 * size_t(kTile) * sizeof(U) + size_t(kWarps) * kRadix * 4 * (kAnyOr ? 2 : 1);
+        return (kTma ? 2 : 1) * size_t(kTile) * sizeof(U) + size_t(kWarps) * kRadix * 4 * (kAnyOr ? 2 : 1);
     }
 };
 
@@ -193,7 +194,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
 
     extern __shared__ __align__(128) unsigned char smem_raw[];
     U* s_in = reinterpret_cast<U*>(smem_raw);                             // TMA-prefetched input tile
-    U* s_keys = s_in + TILE;                                              // digit-ordered staging
+    U* s_keys = Cfg::kTma ? s_in + TILE : s_in;                           // digit-ordered staging
     uint32_t(*s_cnt)[kRadix] = reinterpret_cast<uint32_t(*)[kRadix]>(s_keys + TILE);
     uint32_t(*s_match)[kRadix] = s_cnt + WARPS;  // only touched by atomicOr-ranked items
     __shared__ uint32_t s_delta[kRadix];
@@ -206,7 +207,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     const uint32_t lt = lanemask_lt();
     // the TMA path needs a 16-byte aligned source; full tiles only
     const bool aligned = (reinterpret_cast<uintptr_t>(in) & 15) == 0;
-    auto tma_ok = [&](uint32_t t) { return aligned && uint64_t(t + 1) * TILE <= n; };
+    auto tma_ok = [&](uint32_t t) { return Cfg::kTma && aligned && uint64_t(t + 1) * TILE <= n; };
 
     if (Cfg::kAnyOr) {
         for (int i = tid; i < WARPS * kRadix; i += THREADS) (&s_match[0][0])[i] = 0;
@@ -231,7 +232,14 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
         // --- keys -> registers (warp-striped: warp w owns keys [w*32*ITEMS, (w+1)*32*ITEMS))
         U keys[ITEMS];
         const uint32_t wofs = uint32_t(warp) * 32 * ITEMS + lane;
-        if (tma_ok(tile)) {
+        if (!Cfg::kTma && full) {
+            const U* src = in + tile_base + wofs;
+#pragma unroll
+            for (int i = 0; i < ITEMS; ++i) keys[i] = __ldcs(src + i * 32);
+#pragma unroll
+            for (int i = 0; i < ITEMS; ++i)
+                if (ENC_IN) keys[i] = encode<U, FLOAT>(keys[i]);
+        } else if (tma_ok(tile)) {
             mbar_wait(&s_bar, parity);
             parity ^= 1;
 #pragma unroll
@@ -257,12 +265,6 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
         }
         __syncthreads();  // s_in fully consumed, s_cnt zeroed
 
-        // --- prefetch the next tile into s_in while this one is ranked and scattered
-        if (tid == 0) {
-            const uint32_t nx = atomicAdd(tile_counter, 1u);
-            s_next = nx;
-            if (nx < ntiles && tma_ok(nx)) tma_load_1d(s_in, in + uint64_t(nx) * TILE, TILE * sizeof(U), &s_bar);
-        }
 
         // --- early counts: per-warp digit histogram (fire-and-forget smem adds)
 #pragma unroll
@@ -326,45 +328,67 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
         }
 
         // --- decoupled look-back: exclusive count of digit d over all earlier tiles.
-        // Deferred until after the ranking so predecessors had time to publish;
-        // a 4-wide first probe, then 16-wide windows over runs of aggregates.
+        // Deferred until after the ranking so predecessors had time to publish.
+        // Status word per (tile, digit): flag << 62 | tag << 32 | count; a
+        // window of kLookbackWindow predecessors is read with independent loads,
+        // an unpublished predecessor is then polled alone.
         if (tid < kRadix) {
             const int d = tid;
             uint32_t excl = 0;
             if (tile > 0) {
-                const uint32_t tg = tag & 0x3FFFFFFFu;
-                int64_t t = int64_t(tile) - 1;
+                // high word of a status entry: flag << 30 | tag
+                const uint32_t hi_agg = uint32_t(kFlagAgg << 30) | (tag & 0x3FFFFFFFu);
+                const uint32_t hi_incl = uint32_t(kFlagIncl << 30) | (tag & 0x3FFFFFFFu);
+                uint32_t t = tile - 1;  // newest predecessor not yet consumed
                 const unsigned long long* p = status + uint64_t(t) * kRadix + d;
-                bool done = false;
-                auto probe = [&](auto W) {
-                    constexpr int kW = decltype(W)::value;
-                    unsigned long long w[kW];
+                for (;;) {
+                    // (never below tile 0, which is always inclusive)
+                    uint32_t lo[kLookbackWindow], hi[kLookbackWindow];
 #pragma unroll
-                    for (int k = 0; k < kW; ++k) w[k] = (t - k >= 0) ? ld_relaxed_gpu(p - k * kRadix) : 0ull;
-                    int used = 0;
-#pragma unroll
-                    for (int k = 0; k < kW; ++k) {
-                        if (done || used < k) continue;
-                        const unsigned long long flag = w[k] >> 62;
-                        if (flag == 0 || (uint32_t(w[k] >> 32) & 0x3FFFFFFFu) != tg) continue;  // not published yet
-                        excl += uint32_t(w[k]);
-                        used = k + 1;
-                        if (flag == kFlagIncl) done = true;
+                    for (int k = 0; k < kLookbackWindow; ++k) {
+                        const unsigned long long w = (uint32_t(k) <= t) ? ld_relaxed_gpu(p - k * kRadix) : 0ull;
+                        lo[k] = uint32_t(w);
+                        hi[k] = uint32_t(w >> 32);
                     }
+                    bool go = true, done = false;
+                    uint32_t used = 0;
+#pragma unroll
+                    for (int k = 0; k < kLookbackWindow; ++k) {
+                        const bool ok = hi[k] == hi_agg || hi[k] == hi_incl;
+                        go = go && ok;
+                        if (go) {
+                            excl += lo[k];
+                            ++used;
+                            if (hi[k] == hi_incl) {
+                                done = true;
+                                go = false;
+                            }
+                        }
+                    }
+                    if (done) break;
                     t -= used;
                     p -= used * kRadix;
-                    return used;
-                };
-                int used = probe(std::integral_constant<int, 4>{});
-                while (!done) {
-                    if (used == 0) __nanosleep(64);
-                    used = probe(std::integral_constant<int, 16>{});
+                    if (used == 0) {
+                        unsigned long long w;
+                        do {
+                            __nanosleep(32);
+                            w = ld_relaxed_gpu(p);
+                        } while (uint32_t(w >> 32) != hi_agg && uint32_t(w >> 32) != hi_incl);
+                    }
                 }
                 st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(kFlagIncl, tag, excl + my_total));
             }
             s_delta[d] = base[d] + excl - my_start;
         }
         __syncthreads();
+        if (tid == 0) {
+            // Claim the next tile only now: a tile id claimed earlier would sit
+            // queued behind this tile while its successors wait for its
+            // aggregate.  Its bulk copy (TMA configs) overlaps this scatter.
+            const uint32_t nx = atomicAdd(tile_counter, 1u);
+            s_next = nx;
+            if (nx < ntiles && tma_ok(nx)) tma_load_1d(s_in, in + uint64_t(nx) * TILE, TILE * sizeof(U), &s_bar);
+        }
 
         // --- scatter: consecutive smem slots of one digit go to consecutive output slots
         if (full) {
@@ -389,14 +413,16 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     // no bulk copy is in flight when the block exits
 }
 // Tile configurations (selectable with MSORT_OS_CFG for tuning; 0 = default).
-using Cfg32_0 = OsCfg<384, 20, 0x55555u, 2>;   // alternate ballot / atomicOr (84 KB smem)
-using Cfg32_1 = OsCfg<256, 20, 0xFFFFFu, 4>;   // all ballot, 4 blocks of 256 (48 KB)
-using Cfg32_2 = OsCfg<256, 20, 0x55555u, 3>;   // alternate, 3 blocks of 256 (56 KB)
-using Cfg32_3 = OsCfg<512, 16, 0x5555u, 2>;    // alternate, 2 blocks of 512 (96 KB)
-using Cfg64_0 = OsCfg<384, 12, 0x555u, 2>;
-using Cfg64_1 = OsCfg<256, 12, 0xFFFu, 3>;
-using Cfg64_2 = OsCfg<256, 12, 0x555u, 3>;
-using Cfg64_3 = OsCfg<512, 8, 0x55u, 2>;
+// (measured on B200, profiles/radix_tuning_r1.md: config 0 is the fastest for
+// both key widths; the others stay selectable for tuning)
+using Cfg32_0 = OsCfg<256, 20, 0x55555u, 4, false>;  // alternate ballot / atomicOr, 4 blocks of 256 (36 KB)
+using Cfg32_1 = OsCfg<384, 20, 0x55555u, 2, true>;   // alternate, TMA prefetch (84 KB)
+using Cfg32_2 = OsCfg<256, 20, 0xFFFFFu, 4, true>;   // all ballot, TMA (48 KB)
+using Cfg32_3 = OsCfg<512, 16, 0x5555u, 2, true>;    // alternate, 2 blocks of 512, TMA (96 KB)
+using Cfg64_0 = OsCfg<256, 12, 0x555u, 4, false>;
+using Cfg64_1 = OsCfg<384, 12, 0x555u, 2, true>;
+using Cfg64_2 = OsCfg<256, 12, 0xFFFu, 3, true>;
+using Cfg64_3 = OsCfg<512, 8, 0x55u, 2, true>;
 
 constexpr uint32_t kMinTile32 = 256 * 20;
 constexpr uint32_t kMinTile64 = 256 * 12;  // smallest u64 tile above
@@ -500,6 +526,7 @@ RadixWs radix_ws_layout(void* ws, uint64_t n, int kt) {
     w.head_bytes = head_bytes();
     w.status = reinterpret_cast<unsigned long long*>(p + w.head_bytes);
     w.tiles = (n + radix_tile_keys(kt) - 1) / radix_tile_keys(kt);
+    w.zero_bytes = w.head_bytes + size_t(w.tiles) * kRadix * 8;
     return w;
 }
 
@@ -536,7 +563,7 @@ cudaError_t launch_scan(const uint32_t* hist, uint32_t* base, uint32_t* trivial,
 }
 
 cudaError_t radix_prologue(const void* keys, uint64_t n, int kt, const RadixWs& ws, cudaStream_t st) {
-    cudaError_t e = cudaMemsetAsync(ws.counters, 0, ws.head_bytes + size_t(ws.tiles) * kRadix * 8, st);
+    cudaError_t e = cudaMemsetAsync(ws.counters, 0, ws.zero_bytes, st);
     if (e != cudaSuccess) return e;
     if ((e = launch_histogram(keys, n, kt, ws.hist, st)) != cudaSuccess) return e;
     return launch_scan(ws.hist, ws.base, ws.trivial, n, kt, st);
