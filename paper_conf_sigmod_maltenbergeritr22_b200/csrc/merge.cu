@@ -163,18 +163,200 @@ __global__ void __launch_bounds__(MergeCfg<U>::kThreads) merge_kernel(const U* _
     }
 }
 
+// ---------------------------------------------------------------------------
+// Persistent merge with bulk (TMA) copies: each block walks its output tiles;
+// while tile i is merged from smem, the A and B input ranges of tile i+1 are
+// already streaming into the other smem stage (cp.async.bulk + mbarrier), and
+// the merged tile leaves through a bulk store.  Input ranges start anywhere:
+// the 16-byte aligned body of each range is bulk-copied, the < 16-byte ragged
+// tail is loaded by threads.  Keys stay raw in smem; comparisons use T(key).
+// ---------------------------------------------------------------------------
+struct MergeMeta {
+    uint64_t a0, b0;       // first input key of the tile in a / b
+    int na, nb;            // keys taken from a / b
+    int headA, headB;      // smem slot of key a0 / b0 inside its region
+    int tailA, tailB;      // first smem slot filled by threads (after the bulk body)
+    int ntailA, ntailB;    // keys loaded by threads
+};
+
+template <typename U>
+struct MergeTmaCfg {
+    static constexpr int kThreads = 256;
+    static constexpr int kIpt = sizeof(U) == 4 ? 15 : 7;
+    static constexpr int kTile = kThreads * kIpt;
+    static constexpr int kV = 16 / int(sizeof(U));
+    static constexpr int kRegion = (kTile + 2 * kV + kV - 1) / kV * kV;  // keys per A or B region
+    static constexpr size_t kSmem = size_t(2) * 2 * kRegion * sizeof(U);
+};
+
+__device__ __forceinline__ void bulk_store_1d(void* dst, const void* src, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src)),
+                 "r"(bytes)
+                 : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+
+__device__ __forceinline__ void bulk_wait_read_all() {
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// plan the bulk body / thread tail of one input range [x0, x1) of array `p`
+template <typename U>
+__device__ __forceinline__ uint32_t plan_range(const U* p, uint64_t x0, uint64_t x1, int& head, int& tail,
+                                               int& ntail, const void*& src) {
+    const uintptr_t s = reinterpret_cast<uintptr_t>(p + x0), e = reinterpret_cast<uintptr_t>(p + x1);
+    const uintptr_t as = s & ~uintptr_t(15), ae = e & ~uintptr_t(15);
+    if (x1 <= x0 || ae <= as) {  // no aligned 16-byte unit: everything by threads
+        head = 0;
+        tail = 0;
+        ntail = int(x1 - x0);
+        src = nullptr;
+        return 0;
+    }
+    head = int((s - as) / sizeof(U));
+    tail = int((ae - as) / sizeof(U));
+    ntail = int((e - ae) / sizeof(U));
+    src = reinterpret_cast<const void*>(as);
+    return uint32_t(ae - as);
+}
+
+template <typename U, bool FLOAT>
+__global__ void __launch_bounds__(MergeTmaCfg<U>::kThreads) merge_tma_kernel(const U* __restrict__ a,
+                                                                             const U* __restrict__ b, uint64_t al,
+                                                                             uint64_t bl, U* __restrict__ out,
+                                                                             const uint64_t* __restrict__ part,
+                                                                             uint32_t tiles) {
+    using C = MergeTmaCfg<U>;
+    constexpr int THREADS = C::kThreads, IPT = C::kIpt, TILE = C::kTile, REG = C::kRegion;
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    U* stage = reinterpret_cast<U*>(smem_raw);  // [2 stages][A region | B region]
+    __shared__ MergeMeta meta[2];
+    __shared__ __align__(8) uint64_t bar[2];
+    const int tid = threadIdx.x;
+    const uint64_t total = al + bl;
+
+    auto issue = [&](uint32_t t, int s) {  // thread 0 only
+        const uint64_t k0 = uint64_t(t) * TILE;
+        const uint64_t k1 = k0 + TILE < total ? k0 + TILE : total;
+        const uint64_t a0 = part[t], a1 = part[t + 1];
+        const uint64_t b0 = k0 - a0, b1 = k1 - a1;
+        MergeMeta& m = meta[s];
+        m.a0 = a0;
+        m.b0 = b0;
+        m.na = int(a1 - a0);
+        m.nb = int(b1 - b0);
+        const void *srcA, *srcB;
+        const uint32_t bytesA = plan_range(a, a0, a1, m.headA, m.tailA, m.ntailA, srcA);
+        const uint32_t bytesB = plan_range(b, b0, b1, m.headB, m.tailB, m.ntailB, srcB);
+        U* dA = stage + size_t(s) * 2 * REG;
+        U* dB = dA + REG;
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&bar[s])),
+                     "r"(bytesA + bytesB)
+                     : "memory");
+        if (bytesA)
+            asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                             smem_u32(dA)),
+                         "l"(srcA), "r"(bytesA), "r"(smem_u32(&bar[s]))
+                         : "memory");
+        if (bytesB)
+            asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                             smem_u32(dB)),
+                         "l"(srcB), "r"(bytesB), "r"(smem_u32(&bar[s]))
+                         : "memory");
+    };
+
+    if (tid == 0) {
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
+        if (blockIdx.x < tiles) issue(blockIdx.x, 0);
+    }
+    __syncthreads();
+    uint32_t phase[2] = {0, 0};
+    int s = 0;
+    for (uint32_t t = blockIdx.x; t < tiles; t += gridDim.x, s ^= 1) {
+        const uint32_t tn = t + gridDim.x;
+        if (tid == 0 && tn < tiles) {
+            bulk_wait_read_all();  // the other stage's previous bulk store has left smem
+            issue(tn, s ^ 1);
+        }
+        mbar_wait(&bar[s], phase[s]);
+        phase[s] ^= 1;
+        const MergeMeta m = meta[s];
+        U* sA = stage + size_t(s) * 2 * REG;
+        U* sB = sA + REG;
+        if (tid < m.ntailA) sA[m.tailA + tid] = a[m.a0 - m.headA + m.tailA + tid];
+        if (tid >= 32 && tid - 32 < m.ntailB) sB[m.tailB + tid - 32] = b[m.b0 - m.headB + m.tailB + tid - 32];
+        __syncthreads();
+        const U* xa = sA + m.headA;
+        const U* xb = sB + m.headB;
+        const int na = m.na, nb = m.nb, nt = na + nb;
+        const int d0 = min(tid * IPT, nt);
+        int lo = max(0, d0 - nb), hi = min(d0, na);
+        while (lo < hi) {
+            const int mid = (lo + hi) >> 1;
+            if (encode<U, FLOAT>(xa[mid]) <= encode<U, FLOAT>(xb[d0 - 1 - mid])) lo = mid + 1;
+            else hi = mid;
+        }
+        int ia = lo, ib = d0 - lo;
+        U va = ia < na ? xa[ia] : U(0), vb = ib < nb ? xb[ib] : U(0);
+        U r[IPT];
+#pragma unroll
+        for (int j = 0; j < IPT; ++j) {
+            const bool takeA = ib >= nb || (ia < na && encode<U, FLOAT>(va) <= encode<U, FLOAT>(vb));
+            if (takeA) {
+                r[j] = va;
+                ++ia;
+                va = ia < na ? xa[ia] : U(0);
+            } else {
+                r[j] = vb;
+                ++ib;
+                vb = ib < nb ? xb[ib] : U(0);
+            }
+        }
+        __syncthreads();  // every thread is done reading this stage
+#pragma unroll
+        for (int j = 0; j < IPT; ++j)
+            if (d0 + j < nt) sA[d0 + j] = r[j];
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        __syncthreads();
+        U* dst = out + uint64_t(t) * TILE;
+        const bool bulk = ((reinterpret_cast<uintptr_t>(dst) & 15) == 0) && ((uint32_t(nt) * sizeof(U)) % 16 == 0);
+        if (bulk) {
+            if (tid == 0) bulk_store_1d(dst, sA, uint32_t(nt) * sizeof(U));
+        } else {
+            for (int j = tid; j < nt; j += THREADS) dst[j] = sA[j];
+        }
+        __syncthreads();  // scalar readers of this stage done before it is refilled
+    }
+    if (tid == 0) bulk_wait_all();
+}
+
 template <typename U, bool FLOAT>
 cudaError_t launch_merge_t(const void* a, uint64_t al, const void* b, uint64_t bl, void* out, void* ws,
                            cudaStream_t st, int* launches) {
-    constexpr uint64_t TILE = uint64_t(MergeCfg<U>::kThreads) * MergeCfg<U>::kIpt;
+    using C = MergeTmaCfg<U>;
+    constexpr uint64_t TILE = C::kTile;
     const uint64_t total = al + bl;
     const uint64_t tiles = (total + TILE - 1) / TILE;
     const uint64_t nparts = tiles + 1;
     uint64_t* part = reinterpret_cast<uint64_t*>(ws);
     const unsigned pblocks = unsigned((nparts * 32 + 127) / 128);
     partition_kernel<U, FLOAT><<<pblocks, 128, 0, st>>>((const U*)a, al, (const U*)b, bl, TILE, nparts, part);
-    merge_kernel<U, FLOAT><<<unsigned(tiles), MergeCfg<U>::kThreads, 0, st>>>((const U*)a, (const U*)b, al, bl, (U*)out,
-                                                                            part);
+    auto kern = merge_tma_kernel<U, FLOAT>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(C::kSmem));
+    if (e != cudaSuccess) return e;
+    int per_sm = 0, dev = 0, sms = 0;
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, C::kThreads, C::kSmem)) != cudaSuccess)
+        return e;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    uint64_t grid = uint64_t(per_sm > 0 ? per_sm : 1) * (sms > 0 ? sms : 148);
+    if (grid > tiles) grid = tiles;
+    kern<<<unsigned(grid), C::kThreads, C::kSmem, st>>>((const U*)a, (const U*)b, al, bl, (U*)out, part,
+                                                        uint32_t(tiles));
     if (launches) *launches += 2;
     return cudaGetLastError();
 }
