@@ -50,7 +50,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="msort", choices=["msort", "reference"])
-    ap.add_argument("--n", type=int, default=N_DEFAULT, help="total keys (default 4e9, BASELINE configs[2])")
+    ap.add_argument("--keys", dest="n", type=float, default=N_DEFAULT, help="total keys (default 4e9, BASELINE configs[2])")
     ap.add_argument("--key-type", default="u32")
     ap.add_argument("--dist", default="uniform")
     ap.add_argument("--e2e-steps", type=int, default=3)
@@ -171,6 +171,7 @@ def run_reference(args):
 
 def main():
     args = parse()
+    args.n = int(args.n)
     if args.impl == "reference":
         run_reference(args)
         return
@@ -186,11 +187,17 @@ def main():
     if world != args.gpus:
         if world == 1 and args.gpus > 1:
             raise SystemExit("--gpus N > 1 runs under torchrun (one process per GPU)")
+    # MSORT_BENCH_SAME_GPU=1 maps every rank to cuda:0 (testing the N>1 path on a
+    # one-GPU box: CUDA IPC works between processes on one device)
+    if os.environ.get("MSORT_BENCH_SAME_GPU") == "1":
+        local = 0
     torch.cuda.set_device(local)
     dist = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("cpu:gloo,cuda:nccl", device_id=torch.device("cuda", local))
+        # plumbing only (IPC-handle all-gather, barriers, a max-reduce of the
+        # step times): gloo is enough, the sort itself needs no collective
+        dist.init_process_group("gloo")
     g = world
     kt = args.key_type
     K = mi.KEY_BYTES[kt]
@@ -214,10 +221,8 @@ def main():
         ctx = ms.Context(1, c, kt, device_ids=[local])
         sort_dev = lambda: ctx.sort_device([ms.tensor_ptr(work)], c, streams=[stream])  # noqa: E731
     else:
-        ctx = ms.DistContext(rank, g, local, c, kt)
-        handles = [None] * g
-        dist.all_gather_object(handles, ctx.export_handle())
-        ctx.import_handles(b"".join(handles))
+        from paper_conf_sigmod_maltenbergeritr22_b200 import dist as mdist
+        ctx = mdist.dist_context(rank, g, local, c, kt)
         sort_dev = lambda: ctx.sort(ms.tensor_ptr(work), c, stream=stream)  # noqa: E731
     if args.exchange and g == 1:
         pass

@@ -1,0 +1,104 @@
+"""Parity at BASELINE.json's full sizes, in the launch configurations bench.py
+times, checked by the oracle's any-size properties (oracle/checks.py):
+non-decreasing under T, a permutation of the input (multiset fingerprint), and
+sampled outputs equal to the oracle's order statistics computed one by one.
+Together these imply byte equality with the (unique) oracle result.
+
+configs[2]: 4e9 uniform u32 on one GPU (the bench's N=1 workload);
+configs[1]: 2^28 uniform u32 on 2 chunks (virtual ranks on one GPU);
+configs[3]/[4]: 2e9 keys on 8 chunks (virtual ranks), zipf u32 and f32.
+"""
+import numpy as np
+import pytest
+import torch
+
+import msort_inputs as mi
+from oracle import checks, codec
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+
+BLOCK = 1 << 27
+
+
+def _gen_chunks(n, g, kt, dist, seed):
+    c = n // g
+    chunks = [torch.empty(c, dtype=mi.torch_dtype(kt), device="cuda") for _ in range(g)]
+    for i in range(g):
+        mi.t_generate_into(chunks[i], n, kt, dist, seed=seed, start=i * c, block=BLOCK)
+    return chunks, c
+
+
+def _host_blocks(chunks):
+    for ch in chunks:
+        for off in range(0, ch.numel(), BLOCK):
+            yield ch[off:off + BLOCK].cpu().numpy()
+
+
+def _check(out_chunks, n, kt, dist, seed, nsamples=24):
+    rng = np.random.default_rng(seed)
+    ranks = np.sort(rng.choice(n, size=nsamples, replace=False))
+    ranks[0], ranks[-1] = 0, n - 1
+    # output: sortedness (within and across blocks), fingerprint, sampled values
+    prev = None
+    fp_out = [0, 0, 0]
+    samples = {}
+    pos = 0
+    for blk in _host_blocks(out_chunks):
+        t = codec.encode(blk, kt)
+        assert checks.is_sorted_codes(t), f"not sorted inside block at {pos}"
+        if prev is not None:
+            assert prev <= t[0], f"not sorted across blocks at {pos}"
+        prev = t[-1]
+        f = checks.fingerprint(blk, kt)
+        fp_out = [fp_out[0] + f[0], (fp_out[1] + f[1]) % (1 << 64), fp_out[2] ^ f[2]]
+        for r in ranks[(ranks >= pos) & (ranks < pos + len(blk))]:
+            samples[int(r)] = blk[int(r) - pos]
+        pos += len(blk)
+    assert pos == n
+    # input: fingerprint and order statistics of the sampled outputs, block by block
+    c = n // len(out_chunks)
+    fp_in = [0, 0, 0]
+    sv = codec.encode(np.array([samples[int(r)] for r in ranks], dtype=mi.NP_DTYPE[kt]), kt)
+    lt = np.zeros(len(ranks), dtype=np.int64)
+    le = np.zeros(len(ranks), dtype=np.int64)
+    tmp = torch.empty(BLOCK, dtype=mi.torch_dtype(kt), device="cuda")
+    for off in range(0, n, BLOCK):
+        cnt = min(BLOCK, n - off)
+        mi.t_generate_into(tmp[:cnt], n, kt, dist, seed=seed, start=off, block=BLOCK)
+        blk = tmp[:cnt].cpu().numpy()
+        f = checks.fingerprint(blk, kt)
+        fp_in = [fp_in[0] + f[0], (fp_in[1] + f[1]) % (1 << 64), fp_in[2] ^ f[2]]
+        t = codec.encode(blk, kt)
+        m = len(sv)
+        lt += np.cumsum(np.bincount(np.searchsorted(sv, t, side="right"), minlength=m + 1))[:m]
+        le += np.cumsum(np.bincount(np.searchsorted(sv, t, side="left"), minlength=m + 1))[:m]
+    assert fp_in == fp_out, "output is not a permutation of the input"
+    assert np.all((lt <= ranks) & (ranks < le)), "a sampled output differs from the oracle's order statistic"
+
+
+def test_config3_4e9_u32_one_gpu():
+    import paper_conf_sigmod_maltenbergeritr22_b200 as ms
+    n = 4_000_000_000
+    chunks, c = _gen_chunks(n, 1, "u32", "uniform", 1)
+    ctx = ms.Context(1, n, "u32", device_ids=[0])
+    ctx.sort_device([ms.tensor_ptr(chunks[0])], c)
+    torch.cuda.synchronize()
+    ctx.close()
+    _check(chunks, n, "u32", "uniform", 1)
+
+
+@pytest.mark.parametrize("n,g,kt,dist", [
+    (1 << 28, 2, "u32", "uniform"),          # configs[1]
+    (2_000_000_000, 8, "u32", "zipf"),        # configs[3] (pivot imbalance stress)
+    (2_000_000_000, 8, "f32", "uniform"),     # configs[4] float keys
+])
+def test_p2p_virtual_full_size(n, g, kt, dist):
+    import paper_conf_sigmod_maltenbergeritr22_b200 as ms
+    chunks, c = _gen_chunks(n, g, kt, dist, 3)
+    ctx = ms.Context(g, n, kt, device_ids=[0] * g)
+    ctx.sort_device([ms.tensor_ptr(t) for t in chunks], c)
+    torch.cuda.synchronize()
+    tm = ctx.timings()
+    ctx.close()
+    assert tm["n_stages"] == g - 1
+    _check(chunks, n, kt, dist, 3)
