@@ -123,7 +123,8 @@ int msort_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n);
  * the context's i-th device holding keys_per_gpu keys (16-byte aligned).  On
  * return chunk i holds global ranks [i*c, (i+1)*c) of the union, sorted.
  * streams: NULL or an array of n_gpus cudaStream_t; the sort is ordered after
- * them and they are ordered after the sort.  Blocks until done. */
+ * them (NULL: after each device's legacy default stream) and they are ordered
+ * after the sort.  Blocks until done. */
 int msort_sort_device(msort_ctx* ctx, void* const* chunks, uint64_t keys_per_gpu, void* const* streams);
 
 typedef struct {

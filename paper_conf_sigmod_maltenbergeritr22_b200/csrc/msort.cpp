@@ -739,10 +739,11 @@ int msort_sort_device(msort_ctx* ctx, void* const* chunks, uint64_t keys_per_gpu
                 CUDA_TRY(cudaEventDestroy(e));
                 CUDA_TRY(cudaEventCreate(&e));
             }
-        if (streams && streams[i]) {
-            CUDA_TRY(cudaEventRecord(R.e_sync[MSORT_MAX_STAGES], static_cast<cudaStream_t>(streams[i])));
-            CUDA_TRY(cudaStreamWaitEvent(R.st, R.e_sync[MSORT_MAX_STAGES], 0));
-        }
+        // order the sort after the caller's stream, or after the legacy default
+        // stream when none is given (the context's streams are non-blocking)
+        cudaStream_t us = (streams && streams[i]) ? static_cast<cudaStream_t>(streams[i]) : cudaStreamLegacy;
+        CUDA_TRY(cudaEventRecord(R.e_sync[MSORT_MAX_STAGES], us));
+        CUDA_TRY(cudaStreamWaitEvent(R.st, R.e_sync[MSORT_MAX_STAGES], 0));
     }
     MSORT_TRY(sort_device_local(ctx, keys_per_gpu));
     for (int i = 0; i < ctx->g; ++i)

@@ -8,6 +8,8 @@ configs[2]: 4e9 uniform u32 on one GPU (the bench's N=1 workload);
 configs[1]: 2^28 uniform u32 on 2 chunks (virtual ranks on one GPU);
 configs[3]/[4]: 2e9 keys on 8 chunks (virtual ranks), zipf u32 and f32.
 """
+import os
+
 import numpy as np
 import pytest
 import torch
@@ -34,44 +36,62 @@ def _host_blocks(chunks):
             yield ch[off:off + BLOCK].cpu().numpy()
 
 
+def _block_stats(blk, kt, sv):
+    """Per-block oracle work (numpy releases the GIL: blocks run on a thread pool)."""
+    t = codec.encode(blk, kt)
+    m = len(sv)
+    lt = np.cumsum(np.bincount(np.searchsorted(sv, t, side="right"), minlength=m + 1))[:m]
+    le = np.cumsum(np.bincount(np.searchsorted(sv, t, side="left"), minlength=m + 1))[:m]
+    return checks.fingerprint(blk, kt), lt, le
+
+
+def _out_stats(blk, kt):
+    t = codec.encode(blk, kt)
+    return checks.is_sorted_codes(t), t[0], t[-1], checks.fingerprint(blk, kt)
+
+
+def _fp_add(a, f):
+    return [a[0] + f[0], (a[1] + f[1]) % (1 << 64), a[2] ^ f[2]]
+
+
 def _check(out_chunks, n, kt, dist, seed, nsamples=24):
+    from concurrent.futures import ThreadPoolExecutor
     rng = np.random.default_rng(seed)
     ranks = np.sort(rng.choice(n, size=nsamples, replace=False))
     ranks[0], ranks[-1] = 0, n - 1
+    pool = ThreadPoolExecutor(max_workers=min(16, (os.cpu_count() or 4)))
     # output: sortedness (within and across blocks), fingerprint, sampled values
-    prev = None
-    fp_out = [0, 0, 0]
-    samples = {}
-    pos = 0
+    futs, samples, pos = [], {}, 0
     for blk in _host_blocks(out_chunks):
-        t = codec.encode(blk, kt)
-        assert checks.is_sorted_codes(t), f"not sorted inside block at {pos}"
-        if prev is not None:
-            assert prev <= t[0], f"not sorted across blocks at {pos}"
-        prev = t[-1]
-        f = checks.fingerprint(blk, kt)
-        fp_out = [fp_out[0] + f[0], (fp_out[1] + f[1]) % (1 << 64), fp_out[2] ^ f[2]]
+        futs.append(pool.submit(_out_stats, blk, kt))
         for r in ranks[(ranks >= pos) & (ranks < pos + len(blk))]:
             samples[int(r)] = blk[int(r) - pos]
         pos += len(blk)
     assert pos == n
+    fp_out, prev = [0, 0, 0], None
+    for i, f in enumerate(futs):
+        ok, first, last, fp = f.result()
+        assert ok, f"not sorted inside output block {i}"
+        assert prev is None or prev <= first, f"not sorted across output blocks at {i}"
+        prev = last
+        fp_out = _fp_add(fp_out, fp)
     # input: fingerprint and order statistics of the sampled outputs, block by block
-    c = n // len(out_chunks)
-    fp_in = [0, 0, 0]
     sv = codec.encode(np.array([samples[int(r)] for r in ranks], dtype=mi.NP_DTYPE[kt]), kt)
-    lt = np.zeros(len(ranks), dtype=np.int64)
-    le = np.zeros(len(ranks), dtype=np.int64)
+    futs = []
     tmp = torch.empty(BLOCK, dtype=mi.torch_dtype(kt), device="cuda")
     for off in range(0, n, BLOCK):
         cnt = min(BLOCK, n - off)
         mi.t_generate_into(tmp[:cnt], n, kt, dist, seed=seed, start=off, block=BLOCK)
-        blk = tmp[:cnt].cpu().numpy()
-        f = checks.fingerprint(blk, kt)
-        fp_in = [fp_in[0] + f[0], (fp_in[1] + f[1]) % (1 << 64), fp_in[2] ^ f[2]]
-        t = codec.encode(blk, kt)
-        m = len(sv)
-        lt += np.cumsum(np.bincount(np.searchsorted(sv, t, side="right"), minlength=m + 1))[:m]
-        le += np.cumsum(np.bincount(np.searchsorted(sv, t, side="left"), minlength=m + 1))[:m]
+        futs.append(pool.submit(_block_stats, tmp[:cnt].cpu().numpy(), kt, sv))
+    fp_in = [0, 0, 0]
+    lt = np.zeros(len(ranks), dtype=np.int64)
+    le = np.zeros(len(ranks), dtype=np.int64)
+    for f in futs:
+        fp, a, b = f.result()
+        fp_in = _fp_add(fp_in, fp)
+        lt += a
+        le += b
+    pool.shutdown()
     assert fp_in == fp_out, "output is not a permutation of the input"
     assert np.all((lt <= ranks) & (ranks < le)), "a sampled output differs from the oracle's order statistic"
 
