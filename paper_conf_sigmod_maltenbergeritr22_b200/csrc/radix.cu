@@ -415,16 +415,20 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
 // Tile configurations (selectable with MSORT_OS_CFG for tuning; 0 = default).
 // (measured on B200, profiles/radix_tuning_r1.md: config 0 is the fastest for
 // both key widths; the others stay selectable for tuning)
-using Cfg32_0 = OsCfg<256, 20, 0x55555u, 4, false>;  // alternate ballot / atomicOr, 4 blocks of 256 (36 KB)
-using Cfg32_1 = OsCfg<384, 20, 0x55555u, 2, true>;   // alternate, TMA prefetch (84 KB)
-using Cfg32_2 = OsCfg<256, 20, 0xFFFFFu, 4, true>;   // all ballot, TMA (48 KB)
-using Cfg32_3 = OsCfg<512, 16, 0x5555u, 2, true>;    // alternate, 2 blocks of 512, TMA (96 KB)
-using Cfg64_0 = OsCfg<256, 12, 0x555u, 4, false>;
-using Cfg64_1 = OsCfg<384, 12, 0x555u, 2, true>;
-using Cfg64_2 = OsCfg<256, 12, 0xFFFu, 3, true>;
-using Cfg64_3 = OsCfg<512, 8, 0x55u, 2, true>;
+using Cfg32_0 = OsCfg<256, 28, 0x5555555u, 4, false>;  // 7168-key tiles, 4 blocks of 256 (best, r1)
+using Cfg32_1 = OsCfg<256, 24, 0x555555u, 4, false>;   // 6144-key tiles
+using Cfg32_2 = OsCfg<256, 32, 0x55555555u, 4, false>; // 8192-key tiles
+using Cfg32_3 = OsCfg<256, 28, 0x2492492u, 4, false>;  // 1/3 ballot
+using Cfg32_4 = OsCfg<256, 28, 0x6DB6DB6u, 4, false>;  // 2/3 ballot
+using Cfg32_5 = OsCfg<512, 24, 0x555555u, 2, false>;   // 12288-key tiles, 2 blocks of 512
+using Cfg32_6 = OsCfg<256, 20, 0x55555u, 4, false>;    // previous default
+using Cfg32_7 = OsCfg<384, 20, 0x55555u, 2, true>;     // TMA prefetch (84 KB)
+using Cfg64_0 = OsCfg<256, 14, 0x1555u, 4, false>;
+using Cfg64_1 = OsCfg<256, 12, 0x555u, 4, false>;
+using Cfg64_2 = OsCfg<256, 16, 0x5555u, 4, false>;
+using Cfg64_3 = OsCfg<256, 14, 0x2AAAu, 4, false>;
 
-constexpr uint32_t kMinTile32 = 256 * 20;
+constexpr uint32_t kMinTile32 = 256 * 20;  // smallest u32 tile above
 constexpr uint32_t kMinTile64 = 256 * 12;  // smallest u64 tile above
 
 int env_cfg() {
@@ -432,7 +436,7 @@ int env_cfg() {
     if (v < 0) {
         const char* e = std::getenv("MSORT_OS_CFG");
         v = e ? std::atoi(e) : 0;
-        if (v < 0 || v > 3) v = 0;
+        if (v < 0 || v > 7) v = 0;
     }
     return v;
 }
@@ -475,6 +479,10 @@ cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, c
             case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_1>(in, out, n, pass, ws, base_row, tag, st);
             case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_2>(in, out, n, pass, ws, base_row, tag, st);
             case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_3>(in, out, n, pass, ws, base_row, tag, st);
+            case 4: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_4>(in, out, n, pass, ws, base_row, tag, st);
+            case 5: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_5>(in, out, n, pass, ws, base_row, tag, st);
+            case 6: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_6>(in, out, n, pass, ws, base_row, tag, st);
+            case 7: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_7>(in, out, n, pass, ws, base_row, tag, st);
             default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_0>(in, out, n, pass, ws, base_row, tag, st);
         }
     } else {
@@ -482,6 +490,8 @@ cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, c
             case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_1>(in, out, n, pass, ws, base_row, tag, st);
             case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_2>(in, out, n, pass, ws, base_row, tag, st);
             case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_3>(in, out, n, pass, ws, base_row, tag, st);
+            case 4: case 5: case 6: case 7:
+                return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0>(in, out, n, pass, ws, base_row, tag, st);
             default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0>(in, out, n, pass, ws, base_row, tag, st);
         }
     }

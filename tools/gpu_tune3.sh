@@ -1,0 +1,3 @@
+for cfg in 0 1 2 3 4 5 6 7; do MSORT_OS_CFG=$cfg timeout 300 python tools/time_radix.py 2e9 u32 uniform 3 | cut -c1-200; done
+MSORT_OS_CFG=0 timeout 300 python tools/time_radix.py 2e9 u32 zipf 3 | cut -c1-200
+MSORT_OS_CFG=3 timeout 300 python tools/time_radix.py 2e9 u32 zipf 3 | cut -c1-200
