@@ -109,7 +109,10 @@ enum {
     MSORT_OPT_TIMING = 0,        /* 1: record CUDA events per phase / per radix pass / per merge (default 1) */
     MSORT_OPT_EXCHANGE = 1,      /* 0: fused exchange+merge, the merge kernel loads the partner's block over
                                        NVLink directly (default); 1: swap first (peer copy into a receive
-                                       buffer), then a local merge                              */
+                                       buffer), then a local merge;
+                                       2: NEXT-1, the paper's future work: exact multi-sequence
+                                       splitters over all g sorted chunks, ONE all-to-all exchange (every GPU
+                                       pulls its run from every chunk), local log2(g)-round merge tree       */
     MSORT_OPT_SKIP_TRIVIAL = 2   /* 1: skip radix passes whose digit is constant (identity permutation)   */
 };
 int msort_set_option(msort_ctx* ctx, int option, int64_t value);
@@ -190,6 +193,14 @@ int msort_step_pivot(const void* const* d_chunks, int n_chunks, uint64_t c, int 
 uint64_t msort_merge_workspace_bytes(uint64_t total, int key_type);
 int msort_step_merge(const void* d_a, uint64_t a_len, const void* d_b, uint64_t b_len, void* d_out,
                      int key_type, void* d_ws, uint64_t ws_bytes, void* stream);
+
+/* NEXT-1 splitters (DESIGN reading Q15): for n_chunks sorted
+ * chunks of c keys (HOST array of device pointers, peers allowed) writes the
+ * device uint64 matrix d_s[(n_chunks+1) x n_chunks]: d_s[j*n_chunks + r] = how
+ * many keys of chunk r are among the j*c smallest of the union (ties go to
+ * lower r).  n_chunks in 2..8. */
+int msort_step_splitters(const void* const* d_chunks, int n_chunks, uint64_t c, int key_type, uint64_t* d_s,
+                         void* stream);
 
 /* ------------------------------------------------------------------------ */
 /* Host-side plan (no GPU needed): Alg.2 stage schedule and swap mapping     */

@@ -29,6 +29,7 @@ MSORT_MAX_GPUS = 8
 MSORT_MAX_STAGES = 7
 MSORT_DIST_HANDLE_BYTES = 512
 MSORT_OPT_TIMING, MSORT_OPT_EXCHANGE, MSORT_OPT_SKIP_TRIVIAL = 0, 1, 2
+EXCHANGE_FUSED, EXCHANGE_SWAP, EXCHANGE_ALLTOALL = 0, 1, 2
 MSORT_PASS_ENCODE_IN, MSORT_PASS_DECODE_OUT = 1, 2
 
 STATUS = {0: "MSORT_OK", 1: "MSORT_ERR_INVALID_ARGUMENT", 2: "MSORT_ERR_DEVICE", 3: "MSORT_ERR_OUT_OF_MEMORY",
@@ -38,7 +39,7 @@ EXPORTED = [
     "msort_sort", "msort_create", "msort_destroy", "msort_set_option", "msort_sort_host", "msort_sort_device",
     "msort_get_timings", "msort_status_string", "msort_last_error", "msort_version",
     "msort_radix_workspace_bytes", "msort_step_histogram", "msort_step_radix_pass", "msort_radix_sort",
-    "msort_step_pivot", "msort_merge_workspace_bytes", "msort_step_merge",
+    "msort_step_pivot", "msort_merge_workspace_bytes", "msort_step_merge", "msort_step_splitters",
     "msort_plan_num_stages", "msort_plan_stage", "msort_plan_exchange",
     "msort_dist_create", "msort_dist_export", "msort_dist_import", "msort_dist_sort", "msort_dist_sort_host",
 ]
@@ -105,6 +106,7 @@ _sig("msort_radix_sort", _I, _P, _P, _U64, _I, _P, _U64, _P)
 _sig("msort_step_pivot", _I, ctypes.POINTER(_P), _I, _U64, _I, _P, _P)
 _sig("msort_merge_workspace_bytes", _U64, _U64, _I)
 _sig("msort_step_merge", _I, _P, _U64, _P, _U64, _P, _I, _P, _U64, _P)
+_sig("msort_step_splitters", _I, ctypes.POINTER(_P), _I, _U64, _I, _P, _P)
 _sig("msort_plan_num_stages", _I, _I)
 _sig("msort_plan_stage", _I, _I, _I, ctypes.POINTER(_I))
 _sig("msort_plan_exchange", _I, _I, _I, _U64, ctypes.POINTER(_U64), ctypes.POINTER(_I), ctypes.POINTER(_U64),
@@ -193,6 +195,12 @@ def msort_step_merge(d_a: int, a_len: int, d_b: int, b_len: int, d_out: int, key
                                                      stream_ptr(stream)))
 
 
+def msort_step_splitters(d_chunks: list[int], c: int, key_type, d_s: int, stream=None) -> None:
+    arr = (_P * len(d_chunks))(*d_chunks)
+    _check("msort_step_splitters", _lib.msort_step_splitters(arr, len(d_chunks), c, _kt(key_type), d_s,
+                                                             stream_ptr(stream)))
+
+
 def msort_plan_num_stages(g: int) -> int:
     return _lib.msort_plan_num_stages(g)
 
@@ -271,6 +279,9 @@ class DistContext:
             raise ValueError("need world * MSORT_DIST_HANDLE_BYTES bytes")
         buf = ctypes.create_string_buffer(all_handles, len(all_handles))
         _check("msort_dist_import", _lib.msort_dist_import(self._h, buf))
+
+    def set_option(self, option: int, value: int) -> None:
+        _check("msort_set_option", _lib.msort_set_option(self._h, option, value))
 
     def sort(self, d_chunk: int, c: int, stream=None) -> None:
         _check("msort_dist_sort", _lib.msort_dist_sort(self._h, d_chunk, c, stream_ptr(stream)))

@@ -45,6 +45,9 @@ struct GroupPtrs {
 // of `all`); d_p[j] = pivot of group j.
 cudaError_t launch_pivots(const GroupPtrs& all, int n_groups, int label, uint64_t c, int kt, uint64_t* d_p,
                           cudaStream_t st);
+// NEXT-1 splitters: d_s[j*g + r] (j = 0..g) = keys of chunk r among the j*c
+// smallest of the union of g sorted chunks (all.p[0..g)), ties to lower r.
+cudaError_t launch_splitters(const GroupPtrs& all, int g, uint64_t c, int kt, uint64_t* d_s, cudaStream_t st);
 size_t merge_ws_bytes(uint64_t total, int kt);
 cudaError_t launch_merge(const void* a, uint64_t al, const void* b, uint64_t bl, void* out, int kt, void* ws,
                          cudaStream_t st, int* launches);

@@ -71,6 +71,106 @@ __global__ void __launch_bounds__(32) pivot_kernel(GroupPtrs all, int label, uin
     if (threadIdx.x == 0) p_out[blockIdx.x] = p;
 }
 
+// ---------------------------------------------------------------------------
+// NEXT-1 ("swapping keys between GPUs only once (all-to-all)"):
+// exact multi-sequence splitters.  Block j-1 handles target rank k = j*c over
+// the g sorted chunks (peer pointers): a 32-ary search over the key-code
+// space finds v = the k-th smallest code (each round, warp r counts
+// #{C_r <= candidate} for 32 candidates, one binary search per lane), then the
+// keys equal to v are handed to chunks in index order (DESIGN reading Q15).
+// Output s[j*g + r] = keys of chunk r among the first k (s[0..g) = 0 and
+// s[g*g ..) = c are written by block 0).
+// ---------------------------------------------------------------------------
+template <typename U, bool FLOAT>
+__device__ __forceinline__ uint64_t count_le(const U* p, uint64_t c, U v) {
+    uint64_t lo = 0, hi = c;  // first index with code > v
+    while (lo < hi) {
+        const uint64_t mid = (lo + hi) >> 1;
+        if (encode<U, FLOAT>(p[mid]) <= v) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+template <typename U, bool FLOAT>
+__device__ __forceinline__ uint64_t count_lt(const U* p, uint64_t c, U v) {
+    uint64_t lo = 0, hi = c;  // first index with code >= v
+    while (lo < hi) {
+        const uint64_t mid = (lo + hi) >> 1;
+        if (encode<U, FLOAT>(p[mid]) < v) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+template <typename U, bool FLOAT>
+__global__ void __launch_bounds__(256) splitter_kernel(GroupPtrs all, int g, uint64_t c, uint64_t* s_out) {
+    __shared__ uint64_t cnt[8][32];
+    __shared__ U s_lo, s_hi;
+    __shared__ uint64_t lt_s[8], le_s[8];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint64_t j = blockIdx.x + 1;
+    const uint64_t k = j * c;
+    if (blockIdx.x == 0 && threadIdx.x < 8 && int(threadIdx.x) < g) {
+        s_out[threadIdx.x] = 0;                       // j = 0
+        s_out[uint64_t(g) * g + threadIdx.x] = c;     // j = g
+    }
+    if (threadIdx.x == 0) {
+        s_lo = U(0);
+        s_hi = ~U(0);
+    }
+    __syncthreads();
+    // smallest code v with sum_r #{C_r <= v} >= k   (k <= g*c, so v exists)
+    for (;;) {
+        const U lo = s_lo, hi = s_hi;
+        if (lo >= hi) break;
+        const U step = (hi - lo) / U(32) + U(1);
+        const U span = U(lane) * step;
+        const U cand = (span > hi - lo) ? hi : U(lo + span);
+        if (warp < g) cnt[warp][lane] = count_le<U, FLOAT>(reinterpret_cast<const U*>(all.p[warp]), c, cand);
+        __syncthreads();
+        if (warp == 0) {
+            uint64_t tot = 0;
+            for (int r = 0; r < g; ++r) tot += cnt[r][lane];
+            const uint32_t ok = __ballot_sync(0xffffffffu, tot >= k);
+            if (lane == 0) {
+                // candidates are non-decreasing in lane; lane 31 may be clamped to hi
+                const int f = ok ? __ffs(ok) - 1 : 31;
+                const U cf = (U(f) * step > hi - lo) ? hi : U(lo + U(f) * step);
+                if (!ok) {
+                    // every candidate is below the answer (none was clamped to hi)
+                    s_lo = U(cf + 1);
+                } else if (f == 0) {
+                    s_hi = lo;
+                } else {
+                    const U cp = U(lo + U(f - 1) * step);
+                    s_lo = U(cp + 1);
+                    s_hi = cf;
+                }
+            }
+        }
+        __syncthreads();
+    }
+    const U v = s_lo;
+    if (warp < g && lane == 0) {
+        const U* p = reinterpret_cast<const U*>(all.p[warp]);
+        lt_s[warp] = count_lt<U, FLOAT>(p, c, v);
+        le_s[warp] = count_le<U, FLOAT>(p, c, v);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint64_t lt_tot = 0;
+        for (int r = 0; r < g; ++r) lt_tot += lt_s[r];
+        uint64_t need = k - lt_tot;
+        for (int r = 0; r < g; ++r) {
+            const uint64_t eq = le_s[r] - lt_s[r];
+            const uint64_t take = eq < need ? eq : need;
+            need -= take;
+            s_out[j * g + r] = lt_s[r] + take;
+        }
+    }
+}
+
 template <typename U>
 struct MergeCfg;
 template <>
@@ -400,6 +500,18 @@ cudaError_t launch_pivots(const GroupPtrs& all, int n_groups, int label, uint64_
         case 1: pivot_kernel<uint64_t, false><<<n_groups, 32, 0, st>>>(all, label, c, d_p); break;
         case 2: pivot_kernel<uint32_t, true><<<n_groups, 32, 0, st>>>(all, label, c, d_p); break;
         case 3: pivot_kernel<uint64_t, true><<<n_groups, 32, 0, st>>>(all, label, c, d_p); break;
+        default: return cudaErrorInvalidValue;
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_splitters(const GroupPtrs& all, int g, uint64_t c, int kt, uint64_t* d_s, cudaStream_t st) {
+    const unsigned blocks = unsigned(g > 1 ? g - 1 : 1);
+    switch (kt) {
+        case 0: splitter_kernel<uint32_t, false><<<blocks, 256, 0, st>>>(all, g, c, d_s); break;
+        case 1: splitter_kernel<uint64_t, false><<<blocks, 256, 0, st>>>(all, g, c, d_s); break;
+        case 2: splitter_kernel<uint32_t, true><<<blocks, 256, 0, st>>>(all, g, c, d_s); break;
+        case 3: splitter_kernel<uint64_t, true><<<blocks, 256, 0, st>>>(all, g, c, d_s); break;
         default: return cudaErrorInvalidValue;
     }
     return cudaGetLastError();

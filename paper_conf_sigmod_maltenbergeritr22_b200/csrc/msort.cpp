@@ -133,8 +133,8 @@ struct Rank {
     size_t rws_bytes = 0;
     void* mws = nullptr;
     size_t mws_bytes = 0;
-    uint64_t* d_pivot = nullptr;   // [4]
-    uint64_t* h_pivot = nullptr;   // pinned [4]
+    uint64_t* d_pivot = nullptr;   // [128] pivots (Alg.2) or splitters (all-to-all)
+    uint64_t* h_pivot = nullptr;   // pinned [128]
     uint32_t* h_trivial = nullptr; // pinned [8]
     int* d_err = nullptr;          // barrier timeout flag
     int* h_err = nullptr;          // pinned
@@ -197,10 +197,10 @@ int alloc_rank(msort_ctx* ctx, Rank& R, bool need_b1, bool need_stage) {
     CUDA_TRY(cudaMalloc(&R.rws, R.rws_bytes));
     R.mws_bytes = merge_ws_bytes(ctx->cap, ctx->kt);
     CUDA_TRY(cudaMalloc(&R.mws, R.mws_bytes));
-    CUDA_TRY(cudaMalloc(&R.d_pivot, 8 * sizeof(uint64_t)));
+    CUDA_TRY(cudaMalloc(&R.d_pivot, 128 * sizeof(uint64_t)));
     CUDA_TRY(cudaMalloc(&R.d_err, sizeof(int)));
     CUDA_TRY(cudaMemset(R.d_err, 0, sizeof(int)));
-    CUDA_TRY(cudaMallocHost(&R.h_pivot, 8 * sizeof(uint64_t)));
+    CUDA_TRY(cudaMallocHost(&R.h_pivot, 128 * sizeof(uint64_t)));
     CUDA_TRY(cudaMallocHost(&R.h_trivial, 8 * sizeof(uint32_t)));
     CUDA_TRY(cudaMallocHost(&R.h_err, sizeof(int)));
     *R.h_err = 0;
@@ -363,6 +363,127 @@ void reset_timings(msort_ctx* ctx, uint64_t c) {
 }
 
 // Single-process device-resident sort of r[i].user (c keys each).
+// --- NEXT-1: one all-to-all exchange ----------------------------
+
+// Runs received by rank j: run r = chunk r's keys [s[j][r], s[j+1][r]).
+struct Runs {
+    uint64_t off[MSORT_MAX_GPUS];
+    uint64_t len[MSORT_MAX_GPUS];
+};
+
+Runs runs_of(const uint64_t* s, int g, int j) {
+    Runs rr{};
+    uint64_t o = 0;
+    for (int r = 0; r < g; ++r) {
+        rr.off[r] = o;
+        rr.len[r] = s[(j + 1) * g + r] - s[j * g + r];
+        o += rr.len[r];
+    }
+    return rr;
+}
+
+void record_alltoall_stats(msort_ctx* ctx, const uint64_t* s, int g) {
+    uint64_t mx = 0, sum = 0;
+    for (int j = 0; j < g; ++j) {
+        const Runs rr = runs_of(s, g, j);
+        uint64_t remote = 0;
+        for (int r = 0; r < g; ++r)
+            if (r != j) remote += rr.len[r];
+        mx = std::max(mx, remote);
+        sum += remote;
+    }
+    ctx->tm.n_stages = 1;
+    ctx->tm.stage_label[0] = g;  // one stage over all g chunks
+    ctx->tm.stage_max_x[0] = mx;
+    ctx->tm.stage_keys_exchanged[0] = sum;
+    for (int j = 0; j < g - 1 && j < MSORT_MAX_GPUS / 2; ++j) ctx->tm.stage_pivot[0][j] = 0;
+}
+
+// Multiway merge of the g runs sitting back to back in `src` into `dst_final`,
+// as a tree of two-run merges (log2 g rounds) ping-ponging through `tmp`.
+int merge_tree(msort_ctx* ctx, Rank& R, const Runs& runs, int g, char* src, char* tmp, char* dst_final) {
+    const size_t K = key_bytes(ctx->kt);
+    uint64_t off[MSORT_MAX_GPUS], len[MSORT_MAX_GPUS];
+    int nr = g;
+    for (int r = 0; r < g; ++r) {
+        off[r] = runs.off[r];
+        len[r] = runs.len[r];
+    }
+    char* in = src;
+    char* out = tmp;
+    while (nr > 1) {
+        const bool last = nr == 2;
+        char* o = last ? dst_final : out;
+        int m = 0;
+        for (int i = 0; i + 1 < nr; i += 2) {
+            CUDA_TRY(launch_merge(in + off[i] * K, len[i], in + off[i + 1] * K, len[i + 1], o + off[i] * K, ctx->kt, R.mws,
+                                  R.st, &ctx->tm.kernel_launches));
+            off[m] = off[i];
+            len[m] = len[i] + len[i + 1];
+            ++m;
+        }
+        nr = m;
+        in = o;
+        out = (o == tmp) ? src : tmp;
+    }
+    return MSORT_OK;
+}
+
+int alltoall_local(msort_ctx* ctx, uint64_t c) {
+    const int g = ctx->g;
+    const size_t K = key_bytes(ctx->kt);
+    // every rank's sorted chunk (B1) is complete before anyone reads it
+    for (int i = 0; i < g; ++i) {
+        CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
+        CUDA_TRY(cudaEventRecord(ctx->r[i].e_sync[0], ctx->r[i].st));
+    }
+    for (int i = 0; i < g; ++i) {
+        Rank& R = ctx->r[i];
+        CUDA_TRY(cudaSetDevice(R.dev));
+        for (int q = 0; q < g; ++q)
+            if (q != i) CUDA_TRY(cudaStreamWaitEvent(R.st, ctx->r[q].e_sync[0], 0));
+        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[0][0], R.st));
+    }
+    GroupPtrs all{};
+    for (int i = 0; i < g; ++i) all.p[i] = ctx->r[i].buf[1];
+    Rank& R0 = ctx->r[0];
+    CUDA_TRY(cudaSetDevice(R0.dev));
+    CUDA_TRY(launch_splitters(all, g, c, ctx->kt, R0.d_pivot, R0.st));
+    ctx->tm.kernel_launches += 1;
+    const size_t sbytes = size_t(g + 1) * g * sizeof(uint64_t);
+    CUDA_TRY(cudaMemcpyAsync(R0.h_pivot, R0.d_pivot, sbytes, cudaMemcpyDeviceToHost, R0.st));
+    CUDA_TRY(cudaStreamSynchronize(R0.st));
+    std::vector<uint64_t> s(R0.h_pivot, R0.h_pivot + (g + 1) * g);
+    record_alltoall_stats(ctx, s.data(), g);
+    // the single exchange: rank j pulls its run from every chunk into B0
+    for (int j = 0; j < g; ++j) {
+        Rank& R = ctx->r[j];
+        CUDA_TRY(cudaSetDevice(R.dev));
+        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[0][0], R.st));
+        const Runs rr = runs_of(s.data(), g, j);
+        for (int r = 0; r < g; ++r)
+            if (rr.len[r])
+                CUDA_TRY(cudaMemcpyAsync(static_cast<char*>(R.buf[0]) + rr.off[r] * K,
+                                         static_cast<const char*>(ctx->r[r].buf[1]) + s[j * g + r] * K, rr.len[r] * K,
+                                         cudaMemcpyDefault, R.st));
+        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[0][1], R.st));
+        CUDA_TRY(cudaEventRecord(R.e_sync[1], R.st));
+    }
+    // every pull is done before any B1 is overwritten by a merge round
+    for (int j = 0; j < g; ++j) {
+        Rank& R = ctx->r[j];
+        CUDA_TRY(cudaSetDevice(R.dev));
+        for (int q = 0; q < g; ++q)
+            if (q != j) CUDA_TRY(cudaStreamWaitEvent(R.st, ctx->r[q].e_sync[1], 0));
+        MSORT_TRY(merge_tree(ctx, R, runs_of(s.data(), g, j), g, static_cast<char*>(R.buf[0]),
+                             static_cast<char*>(R.buf[1]), static_cast<char*>(R.user)));
+        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[0][1], R.st));
+        R.cur = -1;
+        CUDA_TRY(cudaEventRecord(R.e_end, R.st));
+    }
+    return MSORT_OK;
+}
+
 int sort_device_local(msort_ctx* ctx, uint64_t c) {
     const int g = ctx->g;
     std::vector<int> labels;
@@ -387,6 +508,7 @@ int sort_device_local(msort_ctx* ctx, uint64_t c) {
         }
         CUDA_TRY(cudaEventRecord(R.e_sorted, R.st));
     }
+    if (g > 1 && ctx->exchange == 2) return alltoall_local(ctx, c);
     const int S = int(labels.size());
     ctx->tm.n_stages = S;
     for (int s = 0; s < S; ++s) {
@@ -596,6 +718,16 @@ int msort_step_pivot(const void* const* d_chunks, int n_chunks, uint64_t c, int 
     return MSORT_OK;
 }
 
+int msort_step_splitters(const void* const* d_chunks, int n_chunks, uint64_t c, int key_type, uint64_t* d_s,
+                         void* stream) {
+    if (!valid_kt(key_type) || !d_chunks || !d_s || n_chunks < 2 || n_chunks > MSORT_MAX_GPUS)
+        return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad argument");
+    GroupPtrs all{};
+    for (int i = 0; i < n_chunks; ++i) all.p[i] = d_chunks[i];
+    CUDA_TRY(launch_splitters(all, n_chunks, c, key_type, d_s, static_cast<cudaStream_t>(stream)));
+    return MSORT_OK;
+}
+
 uint64_t msort_merge_workspace_bytes(uint64_t total, int key_type) {
     if (!valid_kt(key_type)) return 0;
     return merge_ws_bytes(total, key_type);
@@ -677,7 +809,7 @@ int msort_set_option(msort_ctx* ctx, int option, int64_t value) {
         case MSORT_OPT_TIMING: ctx->timing = value ? 1 : 0; return MSORT_OK;
         case MSORT_OPT_SKIP_TRIVIAL: ctx->skip_trivial = value ? 1 : 0; return MSORT_OK;
         case MSORT_OPT_EXCHANGE:
-            if (value != 0 && value != 1) return set_error(MSORT_ERR_INVALID_ARGUMENT, "exchange mode 0 or 1");
+            if (value < 0 || value > 2) return set_error(MSORT_ERR_INVALID_ARGUMENT, "exchange mode 0, 1 or 2");
             if (value == 1)
                 for (int i = 0; i < ctx->nlocal; ++i)
                     if (!ctx->r[i].buf[2]) {
@@ -1051,6 +1183,45 @@ static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* strea
         for (int q = 0; q < g; ++q) cur[q] = 1;
     }
     CUDA_TRY(cudaEventRecord(R.e_sorted, R.st));
+    if (g > 1 && ctx->exchange == 2) {
+        // NEXT-1: splitters from every peer's sorted chunk, one pull per peer,
+        // barrier (peers' B1 no longer read), local merge tree into d_chunk
+        const size_t K = key_bytes(ctx->kt);
+        MSORT_TRY(dist_barrier(ctx));
+        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[0][0], R.st));
+        GroupPtrs all{};
+        for (int q = 0; q < g; ++q) all.p[q] = ctx->peer_buf[q][1];
+        CUDA_TRY(launch_splitters(all, g, c, ctx->kt, R.d_pivot, R.st));
+        ctx->tm.kernel_launches += 1;
+        CUDA_TRY(cudaMemcpyAsync(R.h_pivot, R.d_pivot, size_t(g + 1) * g * sizeof(uint64_t), cudaMemcpyDeviceToHost,
+                                 R.st));
+        CUDA_TRY(cudaMemcpyAsync(R.h_err, R.d_err, sizeof(int), cudaMemcpyDeviceToHost, R.st));
+        CUDA_TRY(cudaStreamSynchronize(R.st));
+        if (*R.h_err) return set_error(MSORT_ERR_TIMEOUT, "device barrier timed out (a peer rank did not arrive)");
+        std::vector<uint64_t> s(R.h_pivot, R.h_pivot + (g + 1) * g);
+        record_alltoall_stats(ctx, s.data(), g);
+        const Runs rr = runs_of(s.data(), g, me);
+        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[0][0], R.st));
+        for (int q = 0; q < g; ++q)
+            if (rr.len[q])
+                CUDA_TRY(cudaMemcpyAsync(static_cast<char*>(R.buf[0]) + rr.off[q] * K,
+                                         static_cast<const char*>(ctx->peer_buf[q][1]) + s[me * g + q] * K, rr.len[q] * K,
+                                         cudaMemcpyDefault, R.st));
+        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[0][1], R.st));
+        MSORT_TRY(dist_barrier(ctx));  // every rank finished pulling from our B1
+        MSORT_TRY(merge_tree(ctx, R, rr, g, static_cast<char*>(R.buf[0]), static_cast<char*>(R.buf[1]),
+                             static_cast<char*>(d_chunk)));
+        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[0][1], R.st));
+        CUDA_TRY(cudaEventRecord(R.e_end, R.st));
+        CUDA_TRY(cudaMemcpyAsync(R.h_err, R.d_err, sizeof(int), cudaMemcpyDeviceToHost, R.st));
+        CUDA_TRY(cudaStreamWaitEvent(ust, R.e_end, 0));
+        CUDA_TRY(cudaStreamSynchronize(R.st));
+        if (*R.h_err) return set_error(MSORT_ERR_TIMEOUT, "device barrier timed out (a peer rank did not arrive)");
+        collect_timings(ctx, 1);
+        collect_exchange_timings(ctx);
+        ctx->tm.total_ms = ctx->tm.sort_ms + ctx->tm.merge_ms;
+        return MSORT_OK;
+    }
     std::vector<int> labels;
     stage_labels(g, labels);
     const int S = int(labels.size());

@@ -263,3 +263,45 @@ def test_errors(ms):
     with pytest.raises(ms.MsortError):
         ms.msort_sort(1234, 10, 9, 1)
     ms.msort_sort(0, 0, "u32", 1)   # n = 0 is a no-op
+
+
+# ---------------------------------------------------------------------------
+# NEXT-1: single all-to-all exchange (MSORT_OPT_EXCHANGE = 2)
+# ---------------------------------------------------------------------------
+
+@pytest.mark.parametrize("g", [2, 4, 8])
+def test_step_splitters(ms, g):
+    rng = np.random.default_rng(g + 100)
+    for trial in range(6):
+        c = int(rng.integers(1, 5000))
+        kt = ["u32", "u64", "f32"][trial % 3]
+        data = mi.np_generate(g * c, kt, "uniform", seed=trial)
+        if kt == "u32" and trial % 2:
+            data = (data % np.uint32(7)).astype(np.uint32)   # heavy ties across chunks
+        chunks = [sort.oracle_sort(data[i * c:(i + 1) * c], kt) for i in range(g)]
+        codes = [codec.encode(x, kt) for x in chunks]
+        expect = [p2p.multiway_splitter(codes, j * c) for j in range(g + 1)]
+        devs = [dev_keys(x) for x in chunks]
+        out = torch.zeros((g + 1) * g, dtype=torch.int64, device="cuda")
+        ms.msort_step_splitters([ms.tensor_ptr(t) for t in devs], c, kt, ms.tensor_ptr(out))
+        torch.cuda.synchronize()
+        got = out.cpu().numpy().reshape(g + 1, g).tolist()
+        assert got == expect, (kt, c)
+
+
+@pytest.mark.parametrize("g", [2, 4, 8])
+@pytest.mark.parametrize("dist", ["uniform", "sorted", "reverse", "zipf", "zipf_rank"])
+def test_alltoall_virtual_ranks(ms, g, dist):
+    c = 3 * 7168 + 52
+    a = mi.np_generate(g * c, "u32", dist, seed=g + 7)
+    out, tm = _virtual_sort(ms, a, "u32", g, exchange=2)
+    assert np.array_equal(out, sort.oracle_sort(a, "u32"))
+    assert tm["n_stages"] == 1 and tm["stage_label"] == [g]
+
+
+@pytest.mark.parametrize("kt", ["u64", "f32", "f64"])
+def test_alltoall_virtual_key_types(ms, kt):
+    g, c = 8, 4001
+    a = mi.np_generate(g * c, kt, "uniform", seed=33)
+    out, _ = _virtual_sort(ms, a, kt, g, exchange=2)
+    assert np.array_equal(bits(out, kt), bits(sort.oracle_sort(a, kt), kt))

@@ -178,3 +178,33 @@ def test_swap_volume_claims(g):
     both = 2 * tot
     expect = (n / 2) * (g - 1)                                  # P:2164-2170, both directions (reading Q12)
     assert abs(both - expect) / expect < {2: 0.1, 4: 0.1, 8: 0.25}[g] * 2
+
+
+def test_multiway_splitter_brute_force():
+    """NEXT-1 splitters (reading Q15): the first s_r keys of every chunk are
+    exactly the k smallest keys of the union; ties go to lower chunks first;
+    monotone in k."""
+    rng = np.random.default_rng(21)
+    for trial in range(400):
+        g = int(rng.choice([2, 3, 4, 8]))
+        c = int(rng.integers(1, 9))
+        hi = int(rng.integers(1, 3 * g * c))
+        chunks = [np.sort(rng.integers(0, hi, c)).astype(np.uint32) for _ in range(g)]
+        union = np.sort(np.concatenate(chunks))
+        prev = [0] * g
+        for k in range(g * c + 1):
+            s = p2p.multiway_splitter(chunks, k)
+            assert sum(s) == k
+            taken = np.concatenate([ch[:sr] for ch, sr in zip(chunks, s)])
+            assert np.array_equal(np.sort(taken), union[:k])
+            assert all(a <= b for a, b in zip(prev, s))
+            prev = s
+            if 0 < k < g * c:
+                v = union[k - 1]
+                # a chunk with an untaken key equal to v: no later chunk took a v
+                for r in range(g):
+                    if s[r] < c and chunks[r][s[r]] == v:
+                        assert all(chunks[q][s[q] - 1] != v for q in range(r + 1, g) if s[q] > 0)
+        out, _ = p2p.alltoall_sort_chunks(chunks)
+        assert np.array_equal(np.concatenate(out), union)
+        assert all(len(o) == c for o in out)
