@@ -1,0 +1,55 @@
+// HET sort baseline (comparison only, never the product path): the CPU side of
+// the paper's heterogeneous sort, §5.3: the g sorted GPU
+// chunks are merged on the host with a parallel multiway merge
+// (gnu_parallel::multiway_merge, a loser tree).  Keys compare by
+// the T order of DESIGN.md reading Q1 (floats: IEEE totalOrder on bits).
+#include <parallel/algorithm>
+#include <omp.h>
+
+#include <cstdint>
+#include <utility>
+#include <vector>
+
+namespace {
+
+template <typename U, bool FLOAT>
+struct TLess {
+    static U code(U u) {
+        if (!FLOAT) return u;
+        constexpr int B = sizeof(U) * 8;
+        const U sign = U(1) << (B - 1);
+        return (u & sign) ? U(~u) : U(u ^ sign);
+    }
+    bool operator()(U a, U b) const { return code(a) < code(b); }
+};
+
+template <typename U, bool FLOAT>
+int merge(const void* const* runs, const uint64_t* lens, int k, void* out, int threads) {
+    using It = U*;  // libstdc++ multiseq_selection wants mutable iterators; inputs are only read
+    std::vector<std::pair<It, It>> seqs;
+    uint64_t total = 0;
+    for (int i = 0; i < k; ++i) {
+        U* p = const_cast<U*>(static_cast<const U*>(runs[i]));
+        seqs.emplace_back(p, p + lens[i]);
+        total += lens[i];
+    }
+    if (threads > 0) omp_set_num_threads(threads);
+    __gnu_parallel::multiway_merge(seqs.begin(), seqs.end(), static_cast<U*>(out), total, TLess<U, FLOAT>(),
+                                   __gnu_parallel::parallel_tag(threads > 0 ? threads : 0));
+    return 0;
+}
+
+}  // namespace
+
+extern "C" int het_multiway_merge(const void* const* runs, const uint64_t* lens, int k, void* out, int key_type,
+                                  int threads) {
+    switch (key_type) {
+        case 0: return merge<uint32_t, false>(runs, lens, k, out, threads);
+        case 1: return merge<uint64_t, false>(runs, lens, k, out, threads);
+        case 2: return merge<uint32_t, true>(runs, lens, k, out, threads);
+        case 3: return merge<uint64_t, true>(runs, lens, k, out, threads);
+        default: return 1;
+    }
+}
+
+extern "C" int het_max_threads() { return omp_get_max_threads(); }

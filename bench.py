@@ -57,7 +57,11 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--seed", type=int, default=1)
-    ap.add_argument("--exchange", type=int, default=0, help="0 fused exchange+merge, 1 swap then merge")
+    ap.add_argument("--exchange", type=int, default=0,
+                    help="merge phase for N>1: 0 the paper's Alg.2 with fused exchange+merge, 1 Alg.2 swap then "
+                         "merge (single process only), 2 NEXT-1 single all-to-all")
+    ap.add_argument("--het", action="store_true", help="also time the HET-sort baseline (GPU chunk sort + CPU merge)")
+    ap.add_argument("--het-chunks", type=int, default=8)
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     return ap.parse_args()
 
@@ -224,10 +228,10 @@ def main():
         from paper_conf_sigmod_maltenbergeritr22_b200 import dist as mdist
         ctx = mdist.dist_context(rank, g, local, c, kt)
         sort_dev = lambda: ctx.sort(ms.tensor_ptr(work), c, stream=stream)  # noqa: E731
-    if args.exchange and g == 1:
-        pass
-    elif args.exchange:
-        raise SystemExit("--exchange 1 is a single-process option")
+    if g > 1:
+        if args.exchange == 1:
+            raise SystemExit("--exchange 1 (swap then merge) is a single-process option")
+        ctx.set_option(ms.MSORT_OPT_EXCHANGE, args.exchange)
 
     def barrier():
         torch.cuda.synchronize()
@@ -323,6 +327,19 @@ def main():
     if rank == 0 and g == 1 and not args.no_cpu:
         cpu = cpu_baseline(n, kt, args.dist, args.seed, args.cpu_seconds)
 
+    het = None
+    if args.het and g == 1:
+        from baseline import het as hetmod
+        hk = pristine[:n].cpu().pin_memory()
+        hetmod.het_sort_host(hk, kt, chunks=args.het_chunks)           # warm-up (allocations, OpenMP start)
+        hk.copy_(pristine[:n].cpu())
+        info = hetmod.het_sort_host(hk, kt, chunks=args.het_chunks)
+        het = {"value": n / info["total_s"], "unit": "keys/s", "kind": "HET sort (paper §5.3): libmsort radix per "
+               f"chunk on 1 GPU + D2H + CPU multiway merge (libstdc++ parallel, {info['threads']} threads)",
+               "chunks": info["chunks"], "gpu_sort_and_copies_s": info["gpu_sort_and_copies_s"],
+               "cpu_merge_s": info["cpu_merge_s"]}
+        del hk
+
     if rank == 0:
         out = {
             "metric": "keys/sec", "value": value, "unit": "keys/s", "n_gpus": g, "steps": args.steps,
@@ -332,7 +349,8 @@ def main():
                                    f"device-resident P2P sort on {g} GPU(s)",
                        "n": n, "keys_per_gpu": c, "key_type": kt, "distribution": args.dist, "seed": args.seed,
                        "parallelism": f"p2p{g}", "l2": "inputs 16 GB >> 126 MB L2 (no flush needed)",
-                       "exchange": "fused peer-read merge" if args.exchange == 0 else "swap then merge"},
+                       "exchange": ["Alg.2, fused peer-read merge", "Alg.2, swap then merge",
+                                    "NEXT-1 single all-to-all"][args.exchange] if g > 1 else "none (1 GPU)"},
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
             "clocks": clk.summary(), "wall_s_timed_region": wall,
             "step_ms": {"min": min(step_ms), "max": max(step_ms)},
@@ -341,6 +359,7 @@ def main():
             "stages": {k: stage_info[k] for k in ("stage_label", "stage_pivot", "stage_max_x", "stage_ms",
                                                   "stage_exchange_ms")} if stage_info and g > 1 else None,
             "paper_context": PAPER_CONTEXT,
+            "het_baseline": het,
         }
         print(json.dumps(out))
     if dist:

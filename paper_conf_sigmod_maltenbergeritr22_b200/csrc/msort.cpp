@@ -144,6 +144,7 @@ struct Rank {
     cudaEvent_t e_sync[MSORT_MAX_STAGES + 1] = {};
     cudaEvent_t e_stage[MSORT_MAX_STAGES][2] = {};
     cudaEvent_t e_xch[MSORT_MAX_STAGES][2] = {};
+    bool xch_rec[MSORT_MAX_STAGES] = {};  // e_xch[s] recorded in this sort
     // per sort
     void* user = nullptr;
     int cur = -1;  // -1: user buffer, 0..2: buf[]
@@ -345,6 +346,7 @@ int launch_exchange(msort_ctx* ctx, Rank& R, int stage, bool last, uint64_t c, u
         }
     }
     if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[stage][1], R.st));
+    R.xch_rec[stage] = ctx->timing != 0;
     new_cur = out_idx;
     return MSORT_OK;
 }
@@ -467,6 +469,7 @@ int alltoall_local(msort_ctx* ctx, uint64_t c) {
                                          static_cast<const char*>(ctx->r[r].buf[1]) + s[j * g + r] * K, rr.len[r] * K,
                                          cudaMemcpyDefault, R.st));
         if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[0][1], R.st));
+        R.xch_rec[0] = ctx->timing != 0;
         CUDA_TRY(cudaEventRecord(R.e_sync[1], R.st));
     }
     // every pull is done before any B1 is overwritten by a merge round
@@ -838,16 +841,14 @@ static int finish_local(msort_ctx* ctx) {
 
 static void collect_exchange_timings(msort_ctx* ctx) {
     if (!ctx->timing) return;
-    // e_xch events are recorded only on ranks that exchanged; query each and
-    // keep the ones that completed (cudaEventElapsedTime fails on unrecorded)
+    // e_xch events are recorded only on ranks that exchanged in that stage
     for (int s = 0; s < ctx->tm.n_stages; ++s) {
         double mx = 0;
         for (int i = 0; i < ctx->nlocal; ++i) {
             Rank& R = ctx->r[i];
+            if (!R.xch_rec[s]) continue;
             cudaSetDevice(R.dev);
-            float ms = 0.f;
-            if (cudaEventElapsedTime(&ms, R.e_xch[s][0], R.e_xch[s][1]) == cudaSuccess) mx = std::max(mx, double(ms));
-            else cudaGetLastError();
+            mx = std::max(mx, double(elapsed(R.e_xch[s][0], R.e_xch[s][1])));
         }
         ctx->tm.stage_exchange_ms[s] = mx;
     }
@@ -866,11 +867,7 @@ int msort_sort_device(msort_ctx* ctx, void* const* chunks, uint64_t keys_per_gpu
         Rank& R = ctx->r[i];
         R.user = chunks[i];
         CUDA_TRY(cudaSetDevice(R.dev));
-        for (int s = 0; s < MSORT_MAX_STAGES; ++s)
-            for (auto& e : R.e_xch[s]) {
-                CUDA_TRY(cudaEventDestroy(e));
-                CUDA_TRY(cudaEventCreate(&e));
-            }
+        for (bool& b : R.xch_rec) b = false;
         // order the sort after the caller's stream, or after the legacy default
         // stream when none is given (the context's streams are non-blocking)
         cudaStream_t us = (streams && streams[i]) ? static_cast<cudaStream_t>(streams[i]) : cudaStreamLegacy;
@@ -904,11 +901,7 @@ int msort_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n) {
     for (int i = 0; i < g; ++i) {
         Rank& R = ctx->r[i];
         CUDA_TRY(cudaSetDevice(R.dev));
-        for (int s = 0; s < MSORT_MAX_STAGES; ++s)
-            for (auto& e : R.e_xch[s]) {
-                CUDA_TRY(cudaEventDestroy(e));
-                CUDA_TRY(cudaEventCreate(&e));
-            }
+        for (bool& b : R.xch_rec) b = false;
         R.user = R.stage;
         const uint64_t lo = std::min<uint64_t>(n, uint64_t(i) * c);
         const uint64_t cnt = std::min<uint64_t>(n - lo, c);
@@ -1160,11 +1153,7 @@ static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* strea
     Rank& R = ctx->r[0];
     CUDA_TRY(cudaSetDevice(R.dev));
     if (!keep_timings) reset_timings(ctx, c);
-    for (int s = 0; s < MSORT_MAX_STAGES; ++s)
-        for (auto& e : R.e_xch[s]) {
-            CUDA_TRY(cudaEventDestroy(e));
-            CUDA_TRY(cudaEventCreate(&e));
-        }
+    for (bool& b : R.xch_rec) b = false;
     cudaStream_t ust = static_cast<cudaStream_t>(stream);
     CUDA_TRY(cudaEventRecord(R.e_sync[MSORT_MAX_STAGES], ust));
     CUDA_TRY(cudaStreamWaitEvent(R.st, R.e_sync[MSORT_MAX_STAGES], 0));
@@ -1208,6 +1197,7 @@ static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* strea
                                          static_cast<const char*>(ctx->peer_buf[q][1]) + s[me * g + q] * K, rr.len[q] * K,
                                          cudaMemcpyDefault, R.st));
         if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[0][1], R.st));
+        R.xch_rec[0] = ctx->timing != 0;
         MSORT_TRY(dist_barrier(ctx));  // every rank finished pulling from our B1
         MSORT_TRY(merge_tree(ctx, R, rr, g, static_cast<char*>(R.buf[0]), static_cast<char*>(R.buf[1]),
                              static_cast<char*>(d_chunk)));
