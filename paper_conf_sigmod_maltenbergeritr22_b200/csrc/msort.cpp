@@ -301,7 +301,8 @@ int radix_passes(msort_ctx* ctx, Rank& R, const void* src, void* dst, void* tmp,
     const void* in = src;
     for (int j = 0; j < E; ++j) {
         void* out = ((E - 1 - j) % 2 == 0) ? dst : tmp;
-        const int flags = (j == 0 ? 1 : 0) | (j == E - 1 ? 2 : 0);
+        // the first executed pass may rank unstably (flag 4): nothing has ordered the keys yet
+        const int flags = (j == 0 ? 1 | 4 : 0) | (j == E - 1 ? 2 : 0);
         if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_pass[j][0], R.st));
         CUDA_TRY(launch_onesweep(in, out, c, ctx->kt, R.pass_ids[j], flags, ws, ws.base + R.pass_ids[j] * 256, R.st));
         ctx->tm.kernel_launches += 1;
@@ -701,7 +702,7 @@ int msort_radix_sort(void* d_keys, void* d_aux, uint64_t n, int key_type, void* 
     for (int p = 0; p < P; ++p) {
         const void* in = (p % 2 == 0) ? d_keys : d_aux;
         void* out = (p % 2 == 0) ? d_aux : d_keys;
-        const int flags = (p == 0 ? 1 : 0) | (p == P - 1 ? 2 : 0);
+        const int flags = (p == 0 ? 1 | 4 : 0) | (p == P - 1 ? 2 : 0);
         CUDA_TRY(launch_onesweep(in, out, n, key_type, p, flags, ws, ws.base + p * 256, st));
     }
     return MSORT_OK;

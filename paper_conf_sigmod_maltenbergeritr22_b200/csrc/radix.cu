@@ -180,7 +180,10 @@ struct OsCfg {
     }
 };
 
-template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg>
+// STABLE = false: ranks within a digit group in arbitrary order (one smem
+// atomic per key, no peer match).  Valid only for the FIRST LSD pass: no
+// earlier pass has ordered the keys, so the order of equal digits is free.
+template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg, bool STABLE = true>
 __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     onesweep_kernel(const U* __restrict__ in, U* __restrict__ out, uint32_t n, uint32_t shift,
                     const uint32_t* __restrict__ base, unsigned long long* __restrict__ status,
@@ -308,6 +311,10 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
 #pragma unroll
         for (int i = 0; i < ITEMS; ++i) {
             const uint32_t d = uint32_t(keys[i] >> shift) & 0xFF;
+            if constexpr (!STABLE) {
+                s_keys[atomicAdd(&s_cnt[warp][d], 1u)] = keys[i];
+                continue;
+            }
             uint32_t peers;
             if ((Cfg::kBallotMask >> i) & 1u) {
                 peers = ballot_match8(d);
@@ -448,11 +455,11 @@ int sm_count() {
     return count > 0 ? count : 148;
 }
 
-template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg>
+template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg, bool STABLE>
 cudaError_t launch_onesweep_c(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
                               const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
     const size_t smem = Cfg::template smem_bytes<U>();
-    auto kern = onesweep_kernel<U, FLOAT, ENC_IN, DEC_OUT, Cfg>;
+    auto kern = onesweep_kernel<U, FLOAT, ENC_IN, DEC_OUT, Cfg, STABLE>;
     // per-device attribute: set on every launch (cheap, and correct when one
     // process drives several GPUs)
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
@@ -470,47 +477,49 @@ cudaError_t launch_onesweep_c(const void* in, void* out, uint64_t n, int pass, c
     return cudaGetLastError();
 }
 
-template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT>
+template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, bool STABLE>
 cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
                               const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
     const int c = env_cfg();
     if constexpr (sizeof(U) == 4) {
         switch (c) {
-            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_1>(in, out, n, pass, ws, base_row, tag, st);
-            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_2>(in, out, n, pass, ws, base_row, tag, st);
-            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_3>(in, out, n, pass, ws, base_row, tag, st);
-            case 4: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_4>(in, out, n, pass, ws, base_row, tag, st);
-            case 5: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_5>(in, out, n, pass, ws, base_row, tag, st);
-            case 6: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_6>(in, out, n, pass, ws, base_row, tag, st);
-            case 7: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_7>(in, out, n, pass, ws, base_row, tag, st);
-            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_0>(in, out, n, pass, ws, base_row, tag, st);
+            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_1, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_2, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_3, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            case 4: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_4, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            case 5: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_5, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            case 6: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_6, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            case 7: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_7, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_0, STABLE>(in, out, n, pass, ws, base_row, tag, st);
         }
     } else {
         switch (c) {
-            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_1>(in, out, n, pass, ws, base_row, tag, st);
-            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_2>(in, out, n, pass, ws, base_row, tag, st);
-            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_3>(in, out, n, pass, ws, base_row, tag, st);
+            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_1, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_2, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_3, STABLE>(in, out, n, pass, ws, base_row, tag, st);
             case 4: case 5: case 6: case 7:
-                return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0>(in, out, n, pass, ws, base_row, tag, st);
-            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0>(in, out, n, pass, ws, base_row, tag, st);
+                return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st);
         }
     }
 }
 
 template <typename U>
-cudaError_t launch_onesweep_int(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
+cudaError_t launch_onesweep_int(const void* in, void* out, uint64_t n, int pass, int flags, const RadixWs& ws,
                                 const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
-    return launch_onesweep_t<U, false, false, false>(in, out, n, pass, ws, base_row, tag, st);
+    if (flags & 4) return launch_onesweep_t<U, false, false, false, false>(in, out, n, pass, ws, base_row, tag, st);
+    return launch_onesweep_t<U, false, false, false, true>(in, out, n, pass, ws, base_row, tag, st);
 }
 
 template <typename U>
 cudaError_t launch_onesweep_float(const void* in, void* out, uint64_t n, int pass, int flags, const RadixWs& ws,
                                   const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
     const bool enc = flags & 1, dec = flags & 2;
-    if (enc && dec) return launch_onesweep_t<U, true, true, true>(in, out, n, pass, ws, base_row, tag, st);
-    if (enc) return launch_onesweep_t<U, true, true, false>(in, out, n, pass, ws, base_row, tag, st);
-    if (dec) return launch_onesweep_t<U, true, false, true>(in, out, n, pass, ws, base_row, tag, st);
-    return launch_onesweep_t<U, true, false, false>(in, out, n, pass, ws, base_row, tag, st);
+    if (enc && dec) return launch_onesweep_t<U, true, true, true, true>(in, out, n, pass, ws, base_row, tag, st);
+    if (enc && (flags & 4)) return launch_onesweep_t<U, true, true, false, false>(in, out, n, pass, ws, base_row, tag, st);
+    if (enc) return launch_onesweep_t<U, true, true, false, true>(in, out, n, pass, ws, base_row, tag, st);
+    if (dec) return launch_onesweep_t<U, true, false, true, true>(in, out, n, pass, ws, base_row, tag, st);
+    return launch_onesweep_t<U, true, false, false, true>(in, out, n, pass, ws, base_row, tag, st);
 }
 
 }  // namespace
@@ -584,8 +593,8 @@ cudaError_t launch_onesweep(const void* in, void* out, uint64_t n, int kt, int p
     if (n == 0) return cudaSuccess;
     const uint32_t tag = uint32_t(pass) + 1;  // status words of other passes are ignored
     switch (kt) {
-        case 0: return launch_onesweep_int<uint32_t>(in, out, n, pass, ws, base_row, tag, st);
-        case 1: return launch_onesweep_int<uint64_t>(in, out, n, pass, ws, base_row, tag, st);
+        case 0: return launch_onesweep_int<uint32_t>(in, out, n, pass, flags, ws, base_row, tag, st);
+        case 1: return launch_onesweep_int<uint64_t>(in, out, n, pass, flags, ws, base_row, tag, st);
         case 2: return launch_onesweep_float<uint32_t>(in, out, n, pass, flags, ws, base_row, tag, st);
         case 3: return launch_onesweep_float<uint64_t>(in, out, n, pass, flags, ws, base_row, tag, st);
         default: return cudaErrorInvalidValue;
