@@ -150,6 +150,10 @@ typedef struct {
 
 int msort_get_timings(const msort_ctx* ctx, msort_timings* out);
 
+/* Ranking used by the onesweep passes on `device`: 1 = one shared-memory atomic
+ * per key (the GPU passed the lane-order self-test, radix.cu), 0 = peer-match
+ * ranking, -1 = no such device. */
+int msort_rank_mode(int device);
 const char* msort_status_string(int status);
 const char* msort_last_error(void);
 int msort_version(void);

@@ -37,7 +37,7 @@ STATUS = {0: "MSORT_OK", 1: "MSORT_ERR_INVALID_ARGUMENT", 2: "MSORT_ERR_DEVICE",
 
 EXPORTED = [
     "msort_sort", "msort_create", "msort_destroy", "msort_set_option", "msort_sort_host", "msort_sort_device",
-    "msort_get_timings", "msort_status_string", "msort_last_error", "msort_version",
+    "msort_get_timings", "msort_status_string", "msort_last_error", "msort_version", "msort_rank_mode",
     "msort_radix_workspace_bytes", "msort_step_histogram", "msort_step_radix_pass", "msort_radix_sort",
     "msort_step_pivot", "msort_merge_workspace_bytes", "msort_step_merge", "msort_step_splitters",
     "msort_plan_num_stages", "msort_plan_stage", "msort_plan_exchange",
@@ -99,6 +99,7 @@ _sig("msort_get_timings", _I, _P, ctypes.POINTER(msort_timings))
 _sig("msort_status_string", ctypes.c_char_p, _I)
 _sig("msort_last_error", ctypes.c_char_p)
 _sig("msort_version", _I)
+_sig("msort_rank_mode", _I, _I)
 _sig("msort_radix_workspace_bytes", _U64, _U64, _I)
 _sig("msort_step_histogram", _I, _P, _U64, _I, _P, _P)
 _sig("msort_step_radix_pass", _I, _P, _P, _U64, _I, _I, _P, _I, _P, _U64, _P)
@@ -160,6 +161,10 @@ def msort_sort(keys: int, n: int, key_type, n_gpus: int = 1, stream=None) -> Non
 
 def msort_version() -> int:
     return _lib.msort_version()
+
+
+def msort_rank_mode(device: int = 0) -> int:
+    return _lib.msort_rank_mode(device)
 
 
 def msort_radix_workspace_bytes(n: int, key_type) -> int:

@@ -33,7 +33,12 @@ cudaError_t radix_prologue(const void* keys, uint64_t n, int kt, const RadixWs& 
 cudaError_t launch_histogram(const void* keys, uint64_t n, int kt, uint32_t* hist, cudaStream_t st);
 // bases from hist rows (all P)
 cudaError_t launch_scan(const uint32_t* hist, uint32_t* base, uint32_t* trivial, uint64_t n, int kt, cudaStream_t st);
-// one onesweep pass; flags: 1 = encode on load, 2 = decode on store
+// true if this GPU serves same-address shared-memory atomics of one warp
+// instruction in lane order (probed once per device; see radix.cu)
+bool atomic_rank_ok();
+// one onesweep pass; flags: 1 = encode on load, 2 = decode on store,
+// 4 = atomic ranking (always valid for the first pass; used for every pass when
+// atomic_rank_ok())
 cudaError_t launch_onesweep(const void* in, void* out, uint64_t n, int kt, int pass, int flags, const RadixWs& ws,
                             const uint32_t* base_row, cudaStream_t st);
 

@@ -189,6 +189,7 @@ namespace {
 int alloc_rank(msort_ctx* ctx, Rank& R, bool need_b1, bool need_stage) {
     const size_t K = key_bytes(ctx->kt);
     CUDA_TRY(cudaSetDevice(R.dev));
+    atomic_rank_ok();  // one-time per-device probe, outside any sort
     CUDA_TRY(cudaStreamCreateWithFlags(&R.st, cudaStreamNonBlocking));
     const size_t bytes = std::max<size_t>(ctx->cap * K, 256);
     CUDA_TRY(cudaMalloc(&R.buf[0], bytes));
@@ -629,6 +630,17 @@ const char* msort_status_string(int status) {
 const char* msort_last_error(void) { return g_last_error.c_str(); }
 
 int msort_version(void) { return 100; }
+
+int msort_rank_mode(int device) {
+    int prev = 0;
+    if (cudaGetDevice(&prev) != cudaSuccess || cudaSetDevice(device) != cudaSuccess) {
+        cudaGetLastError();
+        return -1;
+    }
+    const int r = atomic_rank_ok() ? 1 : 0;
+    cudaSetDevice(prev);
+    return r;
+}
 
 // --- plan ---------------------------------------------------------------------
 

@@ -16,6 +16,7 @@
 //                    coalesced scatter (S3)
 // The float codec T (reading Q1) is applied on the first pass's load and T^-1
 // on the last pass's store (S1), so no separate codec pass touches HBM.
+#include <atomic>
 #include <cstdlib>
 #include <type_traits>
 
@@ -180,9 +181,14 @@ struct OsCfg {
     }
 };
 
-// STABLE = false: ranks within a digit group in arbitrary order (one smem
-// atomic per key, no peer match).  Valid only for the FIRST LSD pass: no
-// earlier pass has ordered the keys, so the order of equal digits is free.
+// STABLE = false: "atomic ranking": each key takes its smem slot with ONE
+// shared-memory atomicAdd on its warp's digit counter (no peer match).  The
+// order in which lanes of one warp instruction that hit the same counter
+// receive their values is not specified by PTX; on sm_100 the hardware serves
+// them in lane order (measured: tools/probe/atom_order.cu), which makes the
+// ranking stable.  atomic_rank_ok() verifies this on the running GPU once per
+// device (rank_probe_kernel) before any stable pass uses it; the first LSD pass
+// may use it regardless (nothing has ordered the keys yet).
 template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg, bool STABLE = true>
 __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     onesweep_kernel(const U* __restrict__ in, U* __restrict__ out, uint32_t n, uint32_t shift,
@@ -448,11 +454,63 @@ int env_cfg() {
     return v;
 }
 
+__global__ void rank_probe_kernel(uint32_t seed, uint32_t* bad);
+
+std::atomic<int> g_rank_ok[64];  // per device: 0 unknown, 1 lane-ordered, -1 not
+
+bool atomic_rank_ok_impl() {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) return false;
+    int v = g_rank_ok[dev].load();
+    if (v != 0) return v > 0;
+    const char* e = std::getenv("MSORT_ATOMIC_RANK");
+    if (e && e[0] == '0') {
+        g_rank_ok[dev] = -1;
+        return false;
+    }
+    uint32_t* bad = nullptr;
+    bool ok = false;
+    if (cudaMalloc(&bad, 4) == cudaSuccess && cudaMemset(bad, 0, 4) == cudaSuccess) {
+        rank_probe_kernel<<<592, 256>>>(0x2545F491u, bad);
+        uint32_t hb = 1;
+        if (cudaMemcpy(&hb, bad, 4, cudaMemcpyDeviceToHost) == cudaSuccess) ok = hb == 0;
+    }
+    if (bad) cudaFree(bad);
+    cudaGetLastError();
+    g_rank_ok[dev] = ok ? 1 : -1;
+    return ok;
+}
+
 int sm_count() {
     int dev = 0, count = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&count, cudaDevAttrMultiProcessorCount, dev);
     return count > 0 ? count : 148;
+}
+
+// Self-test of lane-ordered shared-memory atomics (see STABLE above): random
+// digit patterns of 1..8 bits, warp-private counters, compare every returned
+// value with the match-based stable rank.
+__global__ void __launch_bounds__(256) rank_probe_kernel(uint32_t seed, uint32_t* bad) {
+    __shared__ uint32_t cnt[8][kRadix];
+    const int warp = threadIdx.x >> 5;
+    for (int i = threadIdx.x; i < 8 * kRadix; i += blockDim.x) (&cnt[0][0])[i] = 0;
+    __syncthreads();
+    const uint32_t lt = lanemask_lt();
+    uint32_t h = seed ^ (blockIdx.x * 0x9E3779B9u) ^ (threadIdx.x * 0x85EBCA6Bu);
+    for (int r = 0; r < 256; ++r) {
+        h ^= h << 13;
+        h ^= h >> 17;
+        h ^= h << 5;
+        const uint32_t d = h & ((2u << (r & 7)) - 1u);  // 1..8 significant bits
+        const uint32_t before = cnt[warp][d];
+        __syncwarp();
+        const uint32_t got = atomicAdd(&cnt[warp][d], 1u);
+        const uint32_t want = before + __popc(ballot_match8(d) & lt);
+        if (got != want) atomicAdd(bad, 1u);
+        __syncwarp();
+    }
 }
 
 template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg, bool STABLE>
@@ -515,6 +573,10 @@ template <typename U>
 cudaError_t launch_onesweep_float(const void* in, void* out, uint64_t n, int pass, int flags, const RadixWs& ws,
                                   const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
     const bool enc = flags & 1, dec = flags & 2;
+    const bool atom = flags & 4;
+    if (enc && dec && atom) return launch_onesweep_t<U, true, true, true, false>(in, out, n, pass, ws, base_row, tag, st);
+    if (dec && !enc && atom) return launch_onesweep_t<U, true, false, true, false>(in, out, n, pass, ws, base_row, tag, st);
+    if (!enc && !dec && atom) return launch_onesweep_t<U, true, false, false, false>(in, out, n, pass, ws, base_row, tag, st);
     if (enc && dec) return launch_onesweep_t<U, true, true, true, true>(in, out, n, pass, ws, base_row, tag, st);
     if (enc && (flags & 4)) return launch_onesweep_t<U, true, true, false, false>(in, out, n, pass, ws, base_row, tag, st);
     if (enc) return launch_onesweep_t<U, true, true, false, true>(in, out, n, pass, ws, base_row, tag, st);
@@ -523,6 +585,8 @@ cudaError_t launch_onesweep_float(const void* in, void* out, uint64_t n, int pas
 }
 
 }  // namespace
+
+bool atomic_rank_ok() { return atomic_rank_ok_impl(); }
 
 uint32_t radix_tile_keys(int kt) { return key_bytes(kt) == 4 ? kMinTile32 : kMinTile64; }
 
@@ -592,6 +656,7 @@ cudaError_t launch_onesweep(const void* in, void* out, uint64_t n, int kt, int p
                             const uint32_t* base_row, cudaStream_t st) {
     if (n == 0) return cudaSuccess;
     const uint32_t tag = uint32_t(pass) + 1;  // status words of other passes are ignored
+    if (atomic_rank_ok()) flags |= 4;
     switch (kt) {
         case 0: return launch_onesweep_int<uint32_t>(in, out, n, pass, flags, ws, base_row, tag, st);
         case 1: return launch_onesweep_int<uint64_t>(in, out, n, pass, flags, ws, base_row, tag, st);

@@ -305,3 +305,10 @@ def test_alltoall_virtual_key_types(ms, kt):
     a = mi.np_generate(g * c, kt, "uniform", seed=33)
     out, _ = _virtual_sort(ms, a, kt, g, exchange=2)
     assert np.array_equal(bits(out, kt), bits(sort.oracle_sort(a, kt), kt))
+
+
+def test_rank_mode_probe(ms):
+    # the lane-order self-test ran; report which ranking the passes use
+    mode = ms.msort_rank_mode(0)
+    assert mode in (0, 1)
+    print("onesweep ranking:", "atomic (lane-ordered)" if mode == 1 else "peer match")
