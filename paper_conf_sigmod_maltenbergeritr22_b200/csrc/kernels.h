@@ -16,7 +16,7 @@ struct RadixWs {
     uint32_t* counters;           // [8] per-pass tile counters
     uint32_t* hist;               // [8][256]
     uint32_t* base;               // [8][256] exclusive digit bases
-    uint32_t* trivial;            // [8] 1 if the pass's digit is constant over all keys
+    uint32_t* trivial;            // [8] 1 if the pass's digit is constant over all keys; [8..16) largest bin
     unsigned long long* status;   // [tiles][256] decoupled-lookback words
     uint64_t tiles;
     size_t head_bytes;            // bytes of counters..trivial

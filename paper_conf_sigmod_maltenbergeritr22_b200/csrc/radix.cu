@@ -106,8 +106,12 @@ __global__ void __launch_bounds__(kRadix) scan_kernel(const uint32_t* __restrict
                                                       uint32_t* __restrict__ trivial, uint64_t n) {
     __shared__ uint32_t wsum[kRadix / 32];
     __shared__ int any_full;
+    __shared__ uint32_t max_bin;
     const int p = blockIdx.x, d = threadIdx.x, lane = d & 31, warp = d >> 5;
-    if (d == 0) any_full = 0;
+    if (d == 0) {
+        any_full = 0;
+        max_bin = 0;
+    }
     const uint32_t v = hist[p * kRadix + d];
     uint32_t x = v;
 #pragma unroll
@@ -121,8 +125,12 @@ __global__ void __launch_bounds__(kRadix) scan_kernel(const uint32_t* __restrict
     for (int w = 0; w < warp; ++w) pre += wsum[w];
     base[p * kRadix + d] = pre + x - v;
     if (uint64_t(v) == n) any_full = 1;
+    atomicMax(&max_bin, v);
     __syncthreads();
-    if (d == 0 && trivial) trivial[p] = any_full;
+    if (d == 0 && trivial) {
+        trivial[p] = any_full;
+        trivial[8 + p] = max_bin;  // most frequent digit value of the pass (skew)
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -592,7 +600,7 @@ uint32_t radix_tile_keys(int kt) { return key_bytes(kt) == 4 ? kMinTile32 : kMin
 
 static size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
-static size_t head_bytes() { return align_up(8 * 4 + 8 * 256 * 4 * 2 + 8 * 4, 256); }
+static size_t head_bytes() { return align_up(8 * 4 + 8 * 256 * 4 * 2 + 16 * 4, 256); }
 
 size_t radix_ws_bytes(uint64_t n, int kt) {
     const uint64_t tiles = (n + radix_tile_keys(kt) - 1) / radix_tile_keys(kt);
@@ -656,7 +664,6 @@ cudaError_t launch_onesweep(const void* in, void* out, uint64_t n, int kt, int p
                             const uint32_t* base_row, cudaStream_t st) {
     if (n == 0) return cudaSuccess;
     const uint32_t tag = uint32_t(pass) + 1;  // status words of other passes are ignored
-    if (atomic_rank_ok()) flags |= 4;
     switch (kt) {
         case 0: return launch_onesweep_int<uint32_t>(in, out, n, pass, flags, ws, base_row, tag, st);
         case 1: return launch_onesweep_int<uint64_t>(in, out, n, pass, flags, ws, base_row, tag, st);
