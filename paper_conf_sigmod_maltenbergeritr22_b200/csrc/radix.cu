@@ -147,7 +147,6 @@ __global__ void __launch_bounds__(kRadix) scan_kernel(const uint32_t* __restrict
 // ranking, and the ranking's leader atomicAdd returns the final smem slot.
 // ---------------------------------------------------------------------------
 constexpr unsigned long long kFlagAgg = 1ull, kFlagIncl = 2ull;
-constexpr int kLookbackWindow = 4;
 
 __device__ __forceinline__ unsigned long long pack_status(unsigned long long flag, uint32_t tag, uint32_t count) {
     return (flag << 62) | (uint64_t(tag & 0x3FFFFFFFu) << 32) | count;
@@ -172,9 +171,10 @@ __device__ __forceinline__ uint32_t ballot_match8(uint32_t d) {
 
 // THREADS x ITEMS keys per tile; bit i of BALLOT_MASK: item i ranks with the
 // ballot match (else smem atomicOr); MINB blocks per SM for __launch_bounds__.
-template <int THREADS_, int ITEMS_, uint32_t BALLOT_MASK_, int MINB_, bool TMA_>
+template <int THREADS_, int ITEMS_, uint32_t BALLOT_MASK_, int MINB_, bool TMA_, int LB_ = 4>
 struct OsCfg {
     static constexpr bool kTma = TMA_;  // bulk-copy (TMA) the next tile into smem during the scatter
+    static constexpr int kLookback = LB_;  // look-back window (independent status loads per round)
     static constexpr int kThreads = THREADS_;
     static constexpr int kItems = ITEMS_;
     static constexpr uint32_t kBallotMask = BALLOT_MASK_;
@@ -364,6 +364,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
                 const unsigned long long* p = status + uint64_t(t) * kRadix + d;
                 for (;;) {
                     // (never below tile 0, which is always inclusive)
+                    constexpr int kLookbackWindow = Cfg::kLookback;
                     uint32_t lo[kLookbackWindow], hi[kLookbackWindow];
 #pragma unroll
                     for (int k = 0; k < kLookbackWindow; ++k) {
@@ -436,14 +437,14 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
 // Tile configurations (selectable with MSORT_OS_CFG for tuning; 0 = default).
 // (measured on B200, profiles/radix_tuning_r1.md: config 0 is the fastest for
 // both key widths; the others stay selectable for tuning)
-using Cfg32_0 = OsCfg<256, 28, 0x5555555u, 4, false>;  // 7168-key tiles, 4 blocks of 256 (best, r1)
-using Cfg32_1 = OsCfg<256, 24, 0x555555u, 4, false>;   // 6144-key tiles
-using Cfg32_2 = OsCfg<256, 32, 0x55555555u, 4, false>; // 8192-key tiles
-using Cfg32_3 = OsCfg<256, 28, 0x2492492u, 4, false>;  // 1/3 ballot
-using Cfg32_4 = OsCfg<256, 28, 0x6DB6DB6u, 4, false>;  // 2/3 ballot
-using Cfg32_5 = OsCfg<512, 24, 0x555555u, 2, false>;   // 12288-key tiles, 2 blocks of 512
-using Cfg32_6 = OsCfg<256, 20, 0x55555u, 4, false>;    // previous default
-using Cfg32_7 = OsCfg<384, 20, 0x55555u, 2, true>;     // TMA prefetch (84 KB)
+using Cfg32_0 = OsCfg<256, 28, 0x5555555u, 4, false, 4>;   // 7168-key tiles, 4 blocks of 256 (best, r1)
+using Cfg32_1 = OsCfg<256, 28, 0x5555555u, 4, false, 8>;   // look-back window 8
+using Cfg32_2 = OsCfg<256, 32, 0x55555555u, 4, false, 4>;  // 8192-key tiles
+using Cfg32_3 = OsCfg<256, 24, 0x555555u, 4, false, 4>;    // 6144-key tiles
+using Cfg32_4 = OsCfg<256, 28, 0x5555555u, 3, false, 4>;   // 3 blocks (85 registers)
+using Cfg32_5 = OsCfg<384, 24, 0x555555u, 2, false, 4>;    // 9216-key tiles
+using Cfg32_6 = OsCfg<256, 20, 0x55555u, 4, false, 4>;     // 5120-key tiles
+using Cfg32_7 = OsCfg<384, 20, 0x55555u, 2, true, 4>;      // TMA prefetch (84 KB)
 using Cfg64_0 = OsCfg<256, 14, 0x1555u, 4, false>;
 using Cfg64_1 = OsCfg<256, 12, 0x555u, 4, false>;
 using Cfg64_2 = OsCfg<256, 16, 0x5555u, 4, false>;
