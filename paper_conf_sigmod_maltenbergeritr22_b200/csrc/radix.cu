@@ -171,9 +171,12 @@ __device__ __forceinline__ uint32_t ballot_match8(uint32_t d) {
 
 // THREADS x ITEMS keys per tile; bit i of BALLOT_MASK: item i ranks with the
 // ballot match (else smem atomicOr); MINB blocks per SM for __launch_bounds__.
-template <int THREADS_, int ITEMS_, uint32_t BALLOT_MASK_, int MINB_, bool TMA_, int LB_ = 4>
+template <int THREADS_, int ITEMS_, uint32_t BALLOT_MASK_, int MINB_, bool PF_, int LB_ = 4, bool ELB_ = false,
+          bool CR_ = false>
 struct OsCfg {
-    static constexpr bool kTma = TMA_;  // bulk-copy (TMA) the next tile into smem during the scatter
+    static constexpr bool kCountRank = CR_;  // atomic-ranked passes: rank = the count atomic's return
+    static constexpr bool kEarlyLookback = ELB_;  // look back right after publishing (before the ranking)
+    static constexpr bool kPrefetch = PF_;  // load the next tile's keys into registers during the scatter
     static constexpr int kLookback = LB_;  // look-back window (independent status loads per round)
     static constexpr int kThreads = THREADS_;
     static constexpr int kItems = ITEMS_;
@@ -185,7 +188,7 @@ struct OsCfg {
                                    ((ITEMS_ >= 32 ? 0u : (1u << ITEMS_)) - 1u);
     template <typename U>
     static constexpr size_t smem_bytes() {
-        return (kTma ? 2 : 1) * size_t(kTile) * sizeof(U) + size_t(kWarps) * kRadix * 4 * (kAnyOr ? 2 : 1);
+        return size_t(kTile) * sizeof(U) + size_t(kWarps) * kRadix * 4 * (kAnyOr ? 2 : 1);
     }
 };
 
@@ -197,6 +200,12 @@ struct OsCfg {
 // ranking stable.  atomic_rank_ok() verifies this on the running GPU once per
 // device (rank_probe_kernel) before any stable pass uses it; the first LSD pass
 // may use it regardless (nothing has ordered the keys yet).
+#ifndef MSORT_ABLATE
+#define MSORT_ABLATE 0  // timing ablations (tools/ablate_build.py); never set in a real build
+#endif
+#if MSORT_ABLATE & 8
+__device__ unsigned long long g_lb_stats[4];  // tiles, window rounds, polls, status loads
+#endif
 template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg, bool STABLE = true>
 __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     onesweep_kernel(const U* __restrict__ in, U* __restrict__ out, uint32_t n, uint32_t shift,
@@ -210,86 +219,161 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     static_assert((TILE * sizeof(U)) % 16 == 0, "bulk copies move whole 16-byte units");
 
     extern __shared__ __align__(128) unsigned char smem_raw[];
-    U* s_in = reinterpret_cast<U*>(smem_raw);                             // TMA-prefetched input tile
-    U* s_keys = Cfg::kTma ? s_in + TILE : s_in;                           // digit-ordered staging
+    U* s_keys = reinterpret_cast<U*>(smem_raw);                           // digit-ordered staging
     uint32_t(*s_cnt)[kRadix] = reinterpret_cast<uint32_t(*)[kRadix]>(s_keys + TILE);
     uint32_t(*s_match)[kRadix] = s_cnt + WARPS;  // only touched by atomicOr-ranked items
     __shared__ uint32_t s_delta[kRadix];
     __shared__ uint32_t s_wsum[kRadix / 32];
     __shared__ uint32_t s_next;
-    __shared__ __align__(8) uint64_t s_bar;
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint32_t ntiles = (n + TILE - 1) / TILE;
     const uint32_t lt = lanemask_lt();
-    // the TMA path needs a 16-byte aligned source; full tiles only
-    const bool aligned = (reinterpret_cast<uintptr_t>(in) & 15) == 0;
-    auto tma_ok = [&](uint32_t t) { return Cfg::kTma && aligned && uint64_t(t + 1) * TILE <= n; };
+    const uint32_t wofs = uint32_t(warp) * 32 * ITEMS + lane;
 
-    if (Cfg::kAnyOr) {
-        for (int i = tid; i < WARPS * kRadix; i += THREADS) (&s_match[0][0])[i] = 0;
-    }
-    if (tid == 0) {
-        mbar_init(&s_bar, 1);
-        // Tile ids in arrival order: every lower tile is already held by a
-        // running block, so the look-back below always makes progress.
-        const uint32_t t0 = atomicAdd(tile_counter, 1u);
-        s_next = t0;
-        if (t0 < ntiles && tma_ok(t0)) tma_load_1d(s_in, in + uint64_t(t0) * TILE, TILE * sizeof(U), &s_bar);
-    }
-    __syncthreads();
-    uint32_t parity = 0;
-
-    for (;;) {
-        const uint32_t tile = s_next;
-        if (tile >= ntiles) break;
-        const uint64_t tile_base = uint64_t(tile) * TILE;
-        const bool full = tile_base + TILE <= n;
-
-        // --- keys -> registers (warp-striped: warp w owns keys [w*32*ITEMS, (w+1)*32*ITEMS))
-        U keys[ITEMS];
-        const uint32_t wofs = uint32_t(warp) * 32 * ITEMS + lane;
-        if (!Cfg::kTma && full) {
-            const U* src = in + tile_base + wofs;
+    // keys of tile t -> registers (warp-striped: warp w owns keys [w*32*ITEMS, (w+1)*32*ITEMS)).
+    // Full tiles load raw (encoded by the caller); the partial last tile is
+    // encoded here and its out-of-range slots get the largest code: they rank
+    // after every real key of digit 255 and are never stored (scatter bound).
+    U keys[ITEMS];
+    auto load_tile = [&](uint32_t t) {
+        const uint64_t tb = uint64_t(t) * TILE;
+        const U* src = in + tb + wofs;
+        if (tb + TILE <= n) {
 #pragma unroll
             for (int i = 0; i < ITEMS; ++i) keys[i] = __ldcs(src + i * 32);
-#pragma unroll
-            for (int i = 0; i < ITEMS; ++i)
-                if (ENC_IN) keys[i] = encode<U, FLOAT>(keys[i]);
-        } else if (tma_ok(tile)) {
-            mbar_wait(&s_bar, parity);
-            parity ^= 1;
-#pragma unroll
-            for (int i = 0; i < ITEMS; ++i) keys[i] = s_in[wofs + i * 32];
-#pragma unroll
-            for (int i = 0; i < ITEMS; ++i)
-                if (ENC_IN) keys[i] = encode<U, FLOAT>(keys[i]);
         } else {
-            // out-of-range slots get the largest code: they rank after every real
-            // key of digit 255 and are never stored (see the scatter bound)
-            const U* src = in + tile_base + wofs;
 #pragma unroll
             for (int i = 0; i < ITEMS; ++i) {
-                const bool ok = tile_base + wofs + uint64_t(i) * 32 < n;
+                const bool ok = tb + wofs + uint64_t(i) * 32 < n;
                 U k = ok ? src[i * 32] : U(0);
                 if (ENC_IN) k = encode<U, FLOAT>(k);
                 keys[i] = ok ? k : ~U(0);
             }
         }
+    };
+
+    // --- decoupled look-back: exclusive count of digit d over all earlier tiles.
+    // Status word per (tile, digit): flag << 62 | tag << 32 | count; a window of
+    // kLookback predecessors is read with independent loads, an unpublished
+    // predecessor is then polled alone.  Publishes this tile's inclusive count.
+    auto lookback = [&](const int d, const uint32_t tile, const uint32_t my_total) -> uint32_t {
+        uint32_t excl = 0;
+#if MSORT_ABLATE & 1  // timing ablation: no look-back, uniform-share offsets instead
+        excl = uint32_t(uint64_t(tile) * (n >> 8) / ntiles);
+        if (false) {
+#else
+        if (tile > 0) {
+#endif
+            // high word of a status entry: flag << 30 | tag
+            const uint32_t hi_agg = uint32_t(kFlagAgg << 30) | (tag & 0x3FFFFFFFu);
+            const uint32_t hi_incl = uint32_t(kFlagIncl << 30) | (tag & 0x3FFFFFFFu);
+            uint32_t t = tile - 1;  // newest predecessor not yet consumed
+            const unsigned long long* p = status + uint64_t(t) * kRadix + d;
+            for (;;) {
+                // (never below tile 0, which is always inclusive)
+                constexpr int kLookbackWindow = Cfg::kLookback;
+                uint32_t lo[kLookbackWindow], hi[kLookbackWindow];
+#pragma unroll
+                for (int k = 0; k < kLookbackWindow; ++k) {
+                    const unsigned long long w = (uint32_t(k) <= t) ? ld_relaxed_gpu(p - k * kRadix) : 0ull;
+                    lo[k] = uint32_t(w);
+                    hi[k] = uint32_t(w >> 32);
+                }
+                bool go = true, done = false;
+                uint32_t used = 0;
+#pragma unroll
+                for (int k = 0; k < kLookbackWindow; ++k) {
+                    const bool ok = hi[k] == hi_agg || hi[k] == hi_incl;
+                    go = go && ok;
+                    if (go) {
+                        excl += lo[k];
+                        ++used;
+                        if (hi[k] == hi_incl) {
+                            done = true;
+                            go = false;
+                        }
+                    }
+                }
+#if MSORT_ABLATE & 8
+                atomicAdd(&g_lb_stats[1], 1ull);
+#endif
+                if (done) break;
+                t -= used;
+                p -= used * kRadix;
+                if (used == 0) {
+                    unsigned long long w;
+                    do {
+                        __nanosleep(32);
+#if MSORT_ABLATE & 8
+                        atomicAdd(&g_lb_stats[2], 1ull);
+#endif
+                        w = ld_relaxed_gpu(p);
+                    } while (uint32_t(w >> 32) != hi_agg && uint32_t(w >> 32) != hi_incl);
+                }
+            }
+            st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(kFlagIncl, tag, excl + my_total));
+#if MSORT_ABLATE & 8
+            atomicAdd(&g_lb_stats[0], 1ull);
+#endif
+        }
+        return excl;
+    };
+
+    if (Cfg::kAnyOr) {
+        for (int i = tid; i < WARPS * kRadix; i += THREADS) (&s_match[0][0])[i] = 0;
+    }
+    if (tid == 0) {
+        // Tile ids in arrival order: every lower tile is already held by a
+        // running block, so the look-back below always makes progress.
+        s_next = atomicAdd(tile_counter, 1u);
+    }
+    __syncthreads();
+    uint32_t tile = s_next;
+    if (Cfg::kPrefetch && tile < ntiles) load_tile(tile);
+
+    for (;;) {
+        if (tile >= ntiles) break;
+        const uint64_t tile_base = uint64_t(tile) * TILE;
+        const bool full = tile_base + TILE <= n;
+        if (!Cfg::kPrefetch) load_tile(tile);
+        if (ENC_IN && full) {
+#pragma unroll
+            for (int i = 0; i < ITEMS; ++i) keys[i] = encode<U, FLOAT>(keys[i]);
+        }
         {
             uint4* z = reinterpret_cast<uint4*>(&s_cnt[0][0]);
             for (int i = tid; i < WARPS * kRadix / 4; i += THREADS) z[i] = make_uint4(0, 0, 0, 0);
         }
-        __syncthreads();  // s_in fully consumed, s_cnt zeroed
+        __syncthreads();  // s_cnt zeroed
 
 
-        // --- early counts: per-warp digit histogram (fire-and-forget smem adds)
+        // --- early counts: per-warp digit histogram (fire-and-forget smem adds).
+        // kCountRank (atomic-ranked passes): the count's returned value is the
+        // key's stable rank within (warp, digit) - lane order, see STABLE - kept
+        // as 16-bit halves, so the ranking below is a plain load, not an atomic.
+        constexpr bool kCountRank = Cfg::kCountRank && !STABLE;
+        uint32_t rk[kCountRank ? (ITEMS + 1) / 2 : 1];
+        if constexpr (kCountRank) {
 #pragma unroll
-        for (int i = 0; i < ITEMS; ++i) atomicAdd(&s_cnt[warp][uint32_t(keys[i] >> shift) & 0xFF], 1u);
+            for (int i = 0; i < ITEMS; ++i) {
+                const uint32_t r = atomicAdd(&s_cnt[warp][uint32_t(keys[i] >> shift) & 0xFF], 1u);
+                if (i & 1) rk[i >> 1] |= r << 16;
+                else rk[i >> 1] = r;
+            }
+        } else
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) {
+#if MSORT_ABLATE & 2  // timing ablation only (wrong results): no early counts
+            if (keys[i] == U(0x12345)) 
+#endif
+            atomicAdd(&s_cnt[warp][uint32_t(keys[i] >> shift) & 0xFF], 1u);
+        }
         __syncthreads();
 
         // --- tile totals -> publish aggregate; per-(warp, digit) smem slot bases
         uint32_t my_total = 0, my_start = 0;
+        uint32_t excl_early = 0;
         if (tid < kRadix) {
             const int d = tid;
             uint32_t sum = 0;
@@ -297,6 +381,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
             for (int w = 0; w < WARPS; ++w) sum += s_cnt[w][d];
             my_total = sum;
             st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(tile == 0 ? kFlagIncl : kFlagAgg, tag, sum));
+            if (Cfg::kEarlyLookback) excl_early = lookback(d, tile, sum);
             uint32_t x = sum;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
@@ -325,6 +410,10 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
 #pragma unroll
         for (int i = 0; i < ITEMS; ++i) {
             const uint32_t d = uint32_t(keys[i] >> shift) & 0xFF;
+            if constexpr (kCountRank) {
+                s_keys[s_cnt[warp][d] + ((rk[i >> 1] >> (16 * (i & 1))) & 0xFFFFu)] = keys[i];
+                continue;
+            }
             if constexpr (!STABLE) {
                 s_keys[atomicAdd(&s_cnt[warp][d], 1u)] = keys[i];
                 continue;
@@ -348,68 +437,26 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
             s_keys[slot] = keys[i];
         }
 
-        // --- decoupled look-back: exclusive count of digit d over all earlier tiles.
-        // Deferred until after the ranking so predecessors had time to publish.
-        // Status word per (tile, digit): flag << 62 | tag << 32 | count; a
-        // window of kLookbackWindow predecessors is read with independent loads,
-        // an unpublished predecessor is then polled alone.
+        // --- look-back (deferred until after the ranking unless kEarlyLookback)
         if (tid < kRadix) {
             const int d = tid;
-            uint32_t excl = 0;
-            if (tile > 0) {
-                // high word of a status entry: flag << 30 | tag
-                const uint32_t hi_agg = uint32_t(kFlagAgg << 30) | (tag & 0x3FFFFFFFu);
-                const uint32_t hi_incl = uint32_t(kFlagIncl << 30) | (tag & 0x3FFFFFFFu);
-                uint32_t t = tile - 1;  // newest predecessor not yet consumed
-                const unsigned long long* p = status + uint64_t(t) * kRadix + d;
-                for (;;) {
-                    // (never below tile 0, which is always inclusive)
-                    constexpr int kLookbackWindow = Cfg::kLookback;
-                    uint32_t lo[kLookbackWindow], hi[kLookbackWindow];
-#pragma unroll
-                    for (int k = 0; k < kLookbackWindow; ++k) {
-                        const unsigned long long w = (uint32_t(k) <= t) ? ld_relaxed_gpu(p - k * kRadix) : 0ull;
-                        lo[k] = uint32_t(w);
-                        hi[k] = uint32_t(w >> 32);
-                    }
-                    bool go = true, done = false;
-                    uint32_t used = 0;
-#pragma unroll
-                    for (int k = 0; k < kLookbackWindow; ++k) {
-                        const bool ok = hi[k] == hi_agg || hi[k] == hi_incl;
-                        go = go && ok;
-                        if (go) {
-                            excl += lo[k];
-                            ++used;
-                            if (hi[k] == hi_incl) {
-                                done = true;
-                                go = false;
-                            }
-                        }
-                    }
-                    if (done) break;
-                    t -= used;
-                    p -= used * kRadix;
-                    if (used == 0) {
-                        unsigned long long w;
-                        do {
-                            __nanosleep(32);
-                            w = ld_relaxed_gpu(p);
-                        } while (uint32_t(w >> 32) != hi_agg && uint32_t(w >> 32) != hi_incl);
-                    }
-                }
-                st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(kFlagIncl, tag, excl + my_total));
-            }
+            const uint32_t excl = Cfg::kEarlyLookback ? excl_early : lookback(d, tile, my_total);
             s_delta[d] = base[d] + excl - my_start;
+            // Prefetch configs claim the next tile here so that its loads can
+            // be issued before (and overlap) this tile's scatter.
+            if (Cfg::kPrefetch && tid == 0) s_next = atomicAdd(tile_counter, 1u);
         }
         __syncthreads();
-        if (tid == 0) {
+        if (!Cfg::kPrefetch && tid == 0) {
             // Claim the next tile only now: a tile id claimed earlier would sit
-            // queued behind this tile while its successors wait for its
-            // aggregate.  Its bulk copy (TMA configs) overlaps this scatter.
-            const uint32_t nx = atomicAdd(tile_counter, 1u);
-            s_next = nx;
-            if (nx < ntiles && tma_ok(nx)) tma_load_1d(s_in, in + uint64_t(nx) * TILE, TILE * sizeof(U), &s_bar);
+            // queued behind this tile while its successors wait for its aggregate.
+            s_next = atomicAdd(tile_counter, 1u);
+        }
+        uint32_t next_tile = 0;
+        if (Cfg::kPrefetch) {
+            // keys[] is dead until the next iteration: its loads fly during the scatter
+            next_tile = s_next;
+            if (next_tile < ntiles) load_tile(next_tile);
         }
 
         // --- scatter: consecutive smem slots of one digit go to consecutive output slots
@@ -418,39 +465,40 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
             for (int i = 0; i < ITEMS; ++i) {
                 const uint32_t j = tid + i * THREADS;
                 const U k = s_keys[j];
-                const uint32_t dst = s_delta[uint32_t(k >> shift) & 0xFF] + j;
+                uint32_t dst = s_delta[uint32_t(k >> shift) & 0xFF] + j;
+                if (MSORT_ABLATE) dst = min(dst, n - 1);
                 __stcs(out + dst, DEC_OUT ? decode<U, FLOAT>(k) : k);
             }
         } else {
             const uint32_t valid = uint32_t(n - tile_base);
             for (uint32_t j = tid; j < valid; j += THREADS) {
                 const U k = s_keys[j];
-                const uint32_t dst = s_delta[uint32_t(k >> shift) & 0xFF] + j;
+                uint32_t dst = s_delta[uint32_t(k >> shift) & 0xFF] + j;
+                if (MSORT_ABLATE) dst = min(dst, n - 1);
                 out[dst] = DEC_OUT ? decode<U, FLOAT>(k) : k;
             }
         }
         __syncthreads();
+        tile = Cfg::kPrefetch ? next_tile : s_next;
     }
-    // a prefetch issued for an out-of-range id never happens (guarded above), so
-    // no bulk copy is in flight when the block exits
 }
 // Tile configurations (selectable with MSORT_OS_CFG for tuning; 0 = default).
 // (measured on B200, profiles/radix_tuning_r1.md: config 0 is the fastest for
 // both key widths; the others stay selectable for tuning)
-using Cfg32_0 = OsCfg<256, 28, 0x5555555u, 4, false, 4>;   // 7168-key tiles, 4 blocks of 256 (best, r1)
-using Cfg32_1 = OsCfg<256, 28, 0x5555555u, 4, false, 8>;   // look-back window 8
-using Cfg32_2 = OsCfg<256, 32, 0x55555555u, 4, false, 4>;  // 8192-key tiles
-using Cfg32_3 = OsCfg<256, 24, 0x555555u, 4, false, 4>;    // 6144-key tiles
-using Cfg32_4 = OsCfg<256, 28, 0x5555555u, 3, false, 4>;   // 3 blocks (85 registers)
+using Cfg32_0 = OsCfg<256, 28, 0x5555555u, 4, true, 4>;    // 7168-key tiles, 4 blocks of 256, register prefetch (best)
+using Cfg32_1 = OsCfg<256, 28, 0x5555555u, 4, false, 4>;   // no prefetch (r1 default; 1-2% slower)
+using Cfg32_2 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, true>;  // prefetch + count-rank
+using Cfg32_3 = OsCfg<256, 28, 0x5555555u, 4, true, 4, true>;  // prefetch + look-back before ranking (8% slower)
+using Cfg32_4 = OsCfg<256, 28, 0x5555555u, 4, false, 4, false, true>;  // count-rank
 using Cfg32_5 = OsCfg<384, 24, 0x555555u, 2, false, 4>;    // 9216-key tiles
-using Cfg32_6 = OsCfg<256, 20, 0x55555u, 4, false, 4>;     // 5120-key tiles
-using Cfg32_7 = OsCfg<384, 20, 0x55555u, 2, true, 4>;      // TMA prefetch (84 KB)
-using Cfg64_0 = OsCfg<256, 14, 0x1555u, 4, false>;
+using Cfg32_6 = OsCfg<256, 28, 0x5555555u, 4, false, 4, true>;  // look-back before ranking (9% slower)
+using Cfg32_7 = OsCfg<256, 28, 0x5555555u, 4, true, 8, true>;  // same with window 8 (13% slower)
+using Cfg64_0 = OsCfg<256, 14, 0x1555u, 4, true>;           // register prefetch (best)
 using Cfg64_1 = OsCfg<256, 12, 0x555u, 4, false>;
-using Cfg64_2 = OsCfg<256, 16, 0x5555u, 4, false>;
-using Cfg64_3 = OsCfg<256, 14, 0x2AAAu, 4, false>;
+using Cfg64_2 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, true>;  // prefetch + count-rank
+using Cfg64_3 = OsCfg<256, 14, 0x1555u, 4, false>;          // no prefetch
 
-constexpr uint32_t kMinTile32 = 256 * 20;  // smallest u32 tile above
+constexpr uint32_t kMinTile32 = 256 * 24;  // smallest u32 tile above
 constexpr uint32_t kMinTile64 = 256 * 12;  // smallest u64 tile above
 
 int env_cfg() {
@@ -596,6 +644,17 @@ cudaError_t launch_onesweep_float(const void* in, void* out, uint64_t n, int pas
 }  // namespace
 
 bool atomic_rank_ok() { return atomic_rank_ok_impl(); }
+#if MSORT_ABLATE & 8
+}  // namespace msort
+extern "C" void msort_debug_lb_stats(unsigned long long* out4, int reset) {
+    cudaMemcpyFromSymbol(out4, msort::g_lb_stats, 32);
+    if (reset) {
+        unsigned long long z[4] = {0, 0, 0, 0};
+        cudaMemcpyToSymbol(msort::g_lb_stats, z, 32);
+    }
+}
+namespace msort {
+#endif
 
 uint32_t radix_tile_keys(int kt) { return key_bytes(kt) == 4 ? kMinTile32 : kMinTile64; }
 

@@ -2,6 +2,7 @@
 cfg n kt dist total_ms hist_ms pass_ms_avg GB/s(pass) frac."""
 import os, sys, json
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+if os.environ.get("MSORT_PKG_ROOT"): sys.path.insert(0, os.environ["MSORT_PKG_ROOT"])
 import torch
 import msort_inputs as mi
 import paper_conf_sigmod_maltenbergeritr22_b200 as ms
