@@ -18,9 +18,11 @@ struct RadixWs {
     uint32_t* base;               // [8][256] exclusive digit bases
     uint32_t* trivial;            // [8] 1 if the pass's digit is constant over all keys; [8..16) largest bin
     unsigned long long* status;   // [tiles][256] decoupled-lookback words
+    unsigned long long* gagg;     // [passes][groups][256] look-back group aggregates (tiles << 32 | sum)
     uint64_t tiles;
+    uint64_t groups;
     size_t head_bytes;            // bytes of counters..trivial
-    size_t zero_bytes;            // head + status words: zeroed once per sort
+    size_t zero_bytes;            // head + status words + group aggregates: zeroed once per sort
 };
 uint32_t radix_tile_keys(int kt);
 size_t radix_ws_bytes(uint64_t n, int kt);

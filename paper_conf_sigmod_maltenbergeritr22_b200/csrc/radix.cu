@@ -9,11 +9,12 @@
 //                    lane owns a private smem column per bin, so the smem
 //                    atomics of one warp instruction never collide on a bank
 //   scan_kernel      exclusive prefix per pass -> global digit bases (S2)
-//   onesweep_kernel  persistent blocks; per tile: stable warp ranking (smem
-//                    atomicOr peer masks, or an 8-ballot match), block digit
-//                    counts, decoupled look-back across tiles with a 4-deep
-//                    window for the global digit offset, smem staging,
-//                    coalesced scatter (S3)
+//   onesweep_kernel  persistent blocks; per tile: block digit counts, stable
+//                    warp ranking (lane-ordered smem atomics, or atomicOr /
+//                    8-ballot peer masks), decoupled look-back across tiles
+//                    (windowed, with per-group aggregates) for the global
+//                    digit offset, smem staging, coalesced scatter (S3); the
+//                    next tile's keys load during the scatter
 // The float codec T (reading Q1) is applied on the first pass's load and T^-1
 // on the last pass's store (S1), so no separate codec pass touches HBM.
 #include <atomic>
@@ -172,8 +173,9 @@ __device__ __forceinline__ uint32_t ballot_match8(uint32_t d) {
 // THREADS x ITEMS keys per tile; bit i of BALLOT_MASK: item i ranks with the
 // ballot match (else smem atomicOr); MINB blocks per SM for __launch_bounds__.
 template <int THREADS_, int ITEMS_, uint32_t BALLOT_MASK_, int MINB_, bool PF_, int LB_ = 4, bool ELB_ = false,
-          bool CR_ = false>
+          bool CR_ = false, int GROUP_ = 8>
 struct OsCfg {
+    static constexpr uint32_t kGroup = GROUP_;  // look-back group size (tiles); 0 = tile-by-tile walk only
     static constexpr bool kCountRank = CR_;  // atomic-ranked passes: rank = the count atomic's return
     static constexpr bool kEarlyLookback = ELB_;  // look back right after publishing (before the ranking)
     static constexpr bool kPrefetch = PF_;  // load the next tile's keys into registers during the scatter
@@ -210,7 +212,7 @@ template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg, bool STA
 __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     onesweep_kernel(const U* __restrict__ in, U* __restrict__ out, uint32_t n, uint32_t shift,
                     const uint32_t* __restrict__ base, unsigned long long* __restrict__ status,
-                    uint32_t* __restrict__ tile_counter, uint32_t tag) {
+                    uint32_t* __restrict__ tile_counter, uint32_t tag, unsigned long long* __restrict__ gagg) {
     constexpr int THREADS = Cfg::kThreads;
     constexpr int ITEMS = Cfg::kItems;
     constexpr int WARPS = Cfg::kWarps;
@@ -254,9 +256,14 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     };
 
     // --- decoupled look-back: exclusive count of digit d over all earlier tiles.
-    // Status word per (tile, digit): flag << 62 | tag << 32 | count; a window of
-    // kLookback predecessors is read with independent loads, an unpublished
-    // predecessor is then polled alone.  Publishes this tile's inclusive count.
+    // Status word per (tile, digit): flag << 62 | tag << 32 | count.  Phase 1
+    // walks the predecessors inside this tile's group of kGroup tiles, a window
+    // of kLookback status words per round (an unpublished predecessor is then
+    // polled alone).  Phase 2 walks whole earlier groups: a group contributes
+    // the inclusive count of its last tile if that is published, else its
+    // aggregate word (tiles << 32 | sum, complete when tiles == kGroup; every
+    // tile adds itself right after counting), so a walk of ~30 tiles takes ~3
+    // rounds instead of ~8.  Publishes this tile's inclusive count.
     auto lookback = [&](const int d, const uint32_t tile, const uint32_t my_total) -> uint32_t {
         uint32_t excl = 0;
 #if MSORT_ABLATE & 1  // timing ablation: no look-back, uniform-share offsets instead
@@ -268,24 +275,25 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
             // high word of a status entry: flag << 30 | tag
             const uint32_t hi_agg = uint32_t(kFlagAgg << 30) | (tag & 0x3FFFFFFFu);
             const uint32_t hi_incl = uint32_t(kFlagIncl << 30) | (tag & 0x3FFFFFFFu);
-            uint32_t t = tile - 1;  // newest predecessor not yet consumed
-            const unsigned long long* p = status + uint64_t(t) * kRadix + d;
-            for (;;) {
-                // (never below tile 0, which is always inclusive)
-                constexpr int kLookbackWindow = Cfg::kLookback;
-                uint32_t lo[kLookbackWindow], hi[kLookbackWindow];
+            constexpr int W = Cfg::kLookback;
+            constexpr uint32_t G = Cfg::kGroup;
+            const uint32_t first = G ? tile / (G ? G : 1) * G : 0u;  // phase 1 covers tiles [first, tile)
+            uint32_t left = tile - first;
+            const unsigned long long* p = status + uint64_t(tile - 1) * kRadix + d;
+            bool done = false;
+            while (left > 0) {
+                uint32_t lo[W], hi[W];
 #pragma unroll
-                for (int k = 0; k < kLookbackWindow; ++k) {
-                    const unsigned long long w = (uint32_t(k) <= t) ? ld_relaxed_gpu(p - k * kRadix) : 0ull;
+                for (int k = 0; k < W; ++k) {
+                    const unsigned long long w = uint32_t(k) < left ? ld_relaxed_gpu(p - k * kRadix) : 0ull;
                     lo[k] = uint32_t(w);
                     hi[k] = uint32_t(w >> 32);
                 }
-                bool go = true, done = false;
+                bool go = true;
                 uint32_t used = 0;
 #pragma unroll
-                for (int k = 0; k < kLookbackWindow; ++k) {
-                    const bool ok = hi[k] == hi_agg || hi[k] == hi_incl;
-                    go = go && ok;
+                for (int k = 0; k < W; ++k) {
+                    go = go && (hi[k] == hi_agg || hi[k] == hi_incl);
                     if (go) {
                         excl += lo[k];
                         ++used;
@@ -299,7 +307,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
                 atomicAdd(&g_lb_stats[1], 1ull);
 #endif
                 if (done) break;
-                t -= used;
+                left -= used;  // (tile 0 is always inclusive, so G == 0 ends above)
                 p -= used * kRadix;
                 if (used == 0) {
                     unsigned long long w;
@@ -310,6 +318,50 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
 #endif
                         w = ld_relaxed_gpu(p);
                     } while (uint32_t(w >> 32) != hi_agg && uint32_t(w >> 32) != hi_incl);
+                }
+            }
+            if (G && !done) {
+                uint32_t h = first / (G ? G : 1) - 1;  // newest earlier group not consumed (groups 0..h remain)
+                for (;;) {
+                    uint32_t val[W];
+                    bool ok[W], inc[W];
+#pragma unroll
+                    for (int k = 0; k < W; ++k) {
+                        ok[k] = inc[k] = false;
+                        val[k] = 0;
+                        if (uint32_t(k) <= h) {
+                            const unsigned long long s = ld_relaxed_gpu(status + (uint64_t(h - k + 1) * G - 1) * kRadix + d);
+                            const unsigned long long a = ld_relaxed_gpu(gagg + uint64_t(h - k) * kRadix + d);
+                            inc[k] = uint32_t(s >> 32) == hi_incl;
+                            ok[k] = inc[k] || uint32_t(a >> 32) == G;
+                            val[k] = inc[k] ? uint32_t(s) : uint32_t(a);
+                        }
+                    }
+                    bool go = true;
+                    uint32_t used = 0;
+#pragma unroll
+                    for (int k = 0; k < W; ++k) {
+                        go = go && ok[k];
+                        if (go) {
+                            excl += val[k];
+                            ++used;
+                            if (inc[k]) {
+                                done = true;
+                                go = false;
+                            }
+                        }
+                    }
+#if MSORT_ABLATE & 8
+                    atomicAdd(&g_lb_stats[1], 1ull);
+#endif
+                    if (done || used == h + 1) break;  // (all groups down to 0 consumed)
+                    h -= used;
+                    if (used == 0) {
+#if MSORT_ABLATE & 8
+                        atomicAdd(&g_lb_stats[2], 1ull);
+#endif
+                        __nanosleep(32);
+                    }
                 }
             }
             st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(kFlagIncl, tag, excl + my_total));
@@ -381,6 +433,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
             for (int w = 0; w < WARPS; ++w) sum += s_cnt[w][d];
             my_total = sum;
             st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(tile == 0 ? kFlagIncl : kFlagAgg, tag, sum));
+            if constexpr (Cfg::kGroup != 0) atomicAdd(&gagg[uint64_t(tile / Cfg::kGroup) * kRadix + d], (1ull << 32) | sum);
             if (Cfg::kEarlyLookback) excl_early = lookback(d, tile, sum);
             uint32_t x = sum;
 #pragma unroll
@@ -483,23 +536,26 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     }
 }
 // Tile configurations (selectable with MSORT_OS_CFG for tuning; 0 = default).
-// (measured on B200, profiles/radix_tuning_r1.md: config 0 is the fastest for
-// both key widths; the others stay selectable for tuning)
-using Cfg32_0 = OsCfg<256, 28, 0x5555555u, 4, true, 4>;    // 7168-key tiles, 4 blocks of 256, register prefetch (best)
-using Cfg32_1 = OsCfg<256, 28, 0x5555555u, 4, false, 4>;   // no prefetch (r1 default; 1-2% slower)
-using Cfg32_2 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, true>;  // prefetch + count-rank
-using Cfg32_3 = OsCfg<256, 28, 0x5555555u, 4, true, 4, true>;  // prefetch + look-back before ranking (8% slower)
-using Cfg32_4 = OsCfg<256, 28, 0x5555555u, 4, false, 4, false, true>;  // count-rank
-using Cfg32_5 = OsCfg<384, 24, 0x555555u, 2, false, 4>;    // 9216-key tiles
-using Cfg32_6 = OsCfg<256, 28, 0x5555555u, 4, false, 4, true>;  // look-back before ranking (9% slower)
-using Cfg32_7 = OsCfg<256, 28, 0x5555555u, 4, true, 8, true>;  // same with window 8 (13% slower)
-using Cfg64_0 = OsCfg<256, 14, 0x1555u, 4, true>;           // register prefetch (best)
-using Cfg64_1 = OsCfg<256, 12, 0x555u, 4, false>;
-using Cfg64_2 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, true>;  // prefetch + count-rank
-using Cfg64_3 = OsCfg<256, 14, 0x1555u, 4, false>;          // no prefetch
+// OsCfg<threads, keys/thread, ballot mask, blocks/SM, prefetch, look-back
+// window, look-back before ranking, count-rank, look-back group>; measured on
+// B200 in profiles/radix_tuning_r1.md: config 0 is the fastest for both key
+// widths; the others stay selectable for tuning.
+using Cfg32_0 = OsCfg<256, 28, 0x5555555u, 4, true, 2, false, false, 32>;  // 7168-key tiles, 4 blocks of 256, prefetch,
+                                                                           // look-back window 2, groups of 32 (best)
+using Cfg32_1 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 0>;   // tile-by-tile look-back only
+using Cfg32_2 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 16>;  // look-back groups of 16
+using Cfg32_3 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 64>;  // look-back groups of 64
+using Cfg32_4 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 32>;  // look-back groups of 32
+using Cfg32_5 = OsCfg<256, 28, 0x5555555u, 4, true, 6, false, false, 32>;  // window 6, groups of 32
+using Cfg32_6 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, true>;       // count atomic's return = rank
+using Cfg32_7 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 8>;   // window 4, groups of 8
+using Cfg64_0 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 16>;     // prefetch, groups of 16 (best)
+using Cfg64_1 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 0>;      // tile-by-tile look-back only
+using Cfg64_2 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 8>;      // groups of 8
+using Cfg64_3 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 32>;     // groups of 32
 
-constexpr uint32_t kMinTile32 = 256 * 24;  // smallest u32 tile above
-constexpr uint32_t kMinTile64 = 256 * 12;  // smallest u64 tile above
+constexpr uint32_t kMinTile32 = 256 * 28;  // smallest u32 tile above
+constexpr uint32_t kMinTile64 = 256 * 14;  // smallest u64 tile above
 
 int env_cfg() {
     static int v = -1;
@@ -588,7 +644,7 @@ cudaError_t launch_onesweep_c(const void* in, void* out, uint64_t n, int pass, c
     if (grid > tiles) grid = tiles;
     kern<<<unsigned(grid), Cfg::kThreads, smem, st>>>(reinterpret_cast<const U*>(in), reinterpret_cast<U*>(out),
                                                      uint32_t(n), uint32_t(8 * pass), base_row, ws.status,
-                                                     ws.counters + pass, tag);
+                                                     ws.counters + pass, tag, ws.gagg + size_t(pass) * ws.groups * kRadix);
     return cudaGetLastError();
 }
 
@@ -662,9 +718,14 @@ static size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
 static size_t head_bytes() { return align_up(8 * 4 + 8 * 256 * 4 * 2 + 16 * 4, 256); }
 
+constexpr uint64_t kMinGroup = 8;  // smallest look-back group of the configs above
+
+static uint64_t ws_groups(uint64_t tiles) { return tiles / kMinGroup + 1; }
+
 size_t radix_ws_bytes(uint64_t n, int kt) {
     const uint64_t tiles = (n + radix_tile_keys(kt) - 1) / radix_tile_keys(kt);
-    return head_bytes() + align_up(size_t(tiles) * kRadix * 8, 256) + 256;
+    return head_bytes() + align_up(size_t(tiles) * kRadix * 8, 256) +
+           size_t(num_passes(kt)) * ws_groups(tiles) * kRadix * 8 + 256;
 }
 
 RadixWs radix_ws_layout(void* ws, uint64_t n, int kt) {
@@ -677,7 +738,10 @@ RadixWs radix_ws_layout(void* ws, uint64_t n, int kt) {
     w.head_bytes = head_bytes();
     w.status = reinterpret_cast<unsigned long long*>(p + w.head_bytes);
     w.tiles = (n + radix_tile_keys(kt) - 1) / radix_tile_keys(kt);
-    w.zero_bytes = w.head_bytes + size_t(w.tiles) * kRadix * 8;
+    w.groups = ws_groups(w.tiles);
+    w.gagg = reinterpret_cast<unsigned long long*>(p + w.head_bytes + align_up(size_t(w.tiles) * kRadix * 8, 256));
+    w.zero_bytes = w.head_bytes + align_up(size_t(w.tiles) * kRadix * 8, 256) +
+                   size_t(num_passes(kt)) * w.groups * kRadix * 8;
     return w;
 }
 
