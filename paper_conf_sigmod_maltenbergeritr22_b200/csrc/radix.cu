@@ -426,11 +426,15 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
         // --- tile totals -> publish aggregate; per-(warp, digit) smem slot bases
         uint32_t my_total = 0, my_start = 0;
         uint32_t excl_early = 0;
+        uint32_t col[WARPS];  // this digit's per-warp counts (kept for the slot bases)
         if (tid < kRadix) {
             const int d = tid;
             uint32_t sum = 0;
 #pragma unroll
-            for (int w = 0; w < WARPS; ++w) sum += s_cnt[w][d];
+            for (int w = 0; w < WARPS; ++w) {
+                col[w] = s_cnt[w][d];
+                sum += col[w];
+            }
             my_total = sum;
             st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(tile == 0 ? kFlagIncl : kFlagAgg, tag, sum));
             if constexpr (Cfg::kGroup != 0) atomicAdd(&gagg[uint64_t(tile / Cfg::kGroup) * kRadix + d], (1ull << 32) | sum);
@@ -452,7 +456,8 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
             uint32_t run = my_start;
 #pragma unroll
             for (int w = 0; w < WARPS; ++w) {
-                const uint32_t c = s_cnt[w][tid];
+                // (u64 keys leave no registers to spare: reload instead)
+                const uint32_t c = sizeof(U) == 4 ? col[w] : s_cnt[w][tid];
                 s_cnt[w][tid] = run;
                 run += c;
             }
