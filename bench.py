@@ -75,52 +75,91 @@ def hbm_peak():
 
 
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    """SM clocks and clock-event (throttle) reasons sampled through NVML every
+    ~5 ms in a background thread during the timed region (the first sample is
+    taken before the region opens, so even a 0.2 s region is covered);
+    nvidia-smi is the fallback when NVML is unavailable."""
 
-    def __init__(self, index: int):
+    NAMES = (("hw_slowdown", "nvmlClocksEventReasonHwSlowdown"),
+             ("hw_thermal_slowdown", "nvmlClocksEventReasonHwThermalSlowdown"),
+             ("sw_thermal_slowdown", "nvmlClocksEventReasonSwThermalSlowdown"),
+             ("sw_power_cap", "nvmlClocksEventReasonSwPowerCap"),
+             ("hw_power_brake", "nvmlClocksEventReasonHwPowerBrakeSlowdown"))
+
+    def __init__(self, index: int, pci_bus_id: str | None = None):
         self.index = index
-        self.rows = []
-        self.proc = None
+        self.pci = pci_bus_id
+        self.rows = []  # (sm_mhz, max_mhz, reasons bitmask)
+        self.stop = threading.Event()
+        self.nv = None
+        self.t = None
+
+    def _handle(self):
+        import pynvml as nv
+        nv.nvmlInit()
+        self.nv = nv
+        if self.pci:
+            try:
+                return nv.nvmlDeviceGetHandleByPciBusId(self.pci)
+            except Exception:
+                pass
+        return nv.nvmlDeviceGetHandleByIndex(self.index)
+
+    def _sample(self, h):
+        nv = self.nv
+        sm = nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)
+        mx = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
+        rs = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
+        self.rows.append((float(sm), float(mx), int(rs)))
+
+    def _loop(self, h):
+        while not self.stop.is_set():
+            try:
+                self._sample(h)
+            except Exception:
+                pass
+            self.stop.wait(0.005)
 
     def __enter__(self):
-        q = "clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown," \
-            "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown," \
-            "clocks_event_reasons.sw_power_cap"
         try:
-            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}",
-                                          "--format=csv,noheader,nounits", "-lms", "200"],
-                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-            self.t = threading.Thread(target=self._read, daemon=True)
+            h = self._handle()
+            self._sample(h)
+            self.t = threading.Thread(target=self._loop, args=(h,), daemon=True)
             self.t.start()
         except Exception:
-            self.proc = None
+            self.nv = None
+            self._smi()
         return self
 
-    def _read(self):
-        for line in self.proc.stdout:
-            self.rows.append([x.strip() for x in line.split(",")])
+    def _smi(self):
+        q = "clocks.sm,clocks.max.sm"
+        try:
+            r = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}", "--format=csv,noheader,nounits"],
+                               capture_output=True, text=True, timeout=20)
+            sm, mx = [float(x) for x in r.stdout.strip().split(",")[:2]]
+            self.rows.append((sm, mx, 0))
+        except Exception:
+            pass
 
     def __exit__(self, *a):
-        if self.proc:
-            self.proc.terminate()
-            try:
-                self.proc.wait(timeout=5)
-            except Exception:
-                self.proc.kill()
+        self.stop.set()
+        if self.t:
+            self.t.join(timeout=2)
+        if self.nv is None:
+            self._smi()
 
     def summary(self):
         if not self.rows:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
-        sm = sorted(float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit())
-        mx = max((float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()), default=None)
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        sm = sorted(r[0] for r in self.rows)
         reasons = set()
-        for r in self.rows:
-            for i, nm in enumerate(names):
-                if len(r) > 4 + i and r[4 + i].lower().startswith("active"):
+        if self.nv is not None:
+            for nm, attr in self.NAMES:
+                bit = getattr(self.nv, attr, 0)
+                if any(r[2] & bit for r in self.rows):
                     reasons.add(nm)
-        return {"sm_mhz": sm[len(sm) // 2] if sm else None, "sm_max_mhz": mx, "reasons": sorted(reasons),
-                "samples": len(self.rows)}
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": max(r[1] for r in self.rows), "reasons": sorted(reasons),
+                "samples": len(self.rows), "source": "nvml" if self.nv is not None else "nvidia-smi"}
 
 
 def cpu_baseline(n_total: int, key_type: str, dist: str, seed: int, seconds: float):
@@ -247,7 +286,12 @@ def main():
     barrier()
     pass_ms, pass_cnt, stage_info, launches = 0.0, 0, None, 0
     hist_ms = 0.0
-    with ClockSampler(local) as clk:
+    try:
+        pp = torch.cuda.get_device_properties(dev)
+        pci = f"{pp.pci_domain_id:08X}:{pp.pci_bus_id:02X}:{pp.pci_device_id:02X}.0"
+    except Exception:
+        pci = None
+    with ClockSampler(local, pci) as clk:
         barrier()
         t_wall = time.perf_counter()
         for i in range(args.steps):
