@@ -17,6 +17,8 @@
 //   fill_kernel    tail padding with the largest key (reading Q3).
 //   barrier_kernel device-side barrier over IPC-mapped flags (dist mode).
 // All comparisons are on T(key) (reading Q1), so floats order by totalOrder.
+#include <cstdlib>
+
 #include "common.cuh"
 #include "kernels.h"
 
@@ -200,6 +202,27 @@ __global__ void __launch_bounds__(128) partition_kernel(const U* __restrict__ a,
         return encode<U, FLOAT>(a[i]) <= encode<U, FLOAT>(b[k - 1 - i]);
     });
     if ((threadIdx.x & 31) == 0) part[w] = r;
+}
+
+// Same partition, one THREAD per boundary (plain binary search): the top levels
+// of all searches hit the same L2 lines, so DRAM sees only the last few levels
+// of each search (the warp version above touches 64 sectors per round).
+template <typename U, bool FLOAT>
+__global__ void __launch_bounds__(256) partition_thread_kernel(const U* __restrict__ a, uint64_t al,
+                                                               const U* __restrict__ b, uint64_t bl, uint64_t tile,
+                                                               uint64_t nparts, uint64_t* __restrict__ part) {
+    const uint64_t w = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (w >= nparts) return;
+    const uint64_t total = al + bl;
+    const uint64_t k = w * tile < total ? w * tile : total;
+    uint64_t lo = k > bl ? k - bl : 0;
+    uint64_t hi = k < al ? k : al;
+    while (lo < hi) {
+        const uint64_t mid = (lo + hi) >> 1;
+        if (encode<U, FLOAT>(a[mid]) <= encode<U, FLOAT>(b[k - 1 - mid])) lo = mid + 1;
+        else hi = mid;
+    }
+    part[w] = lo;
 }
 
 // Block merge of one output tile: stage both input ranges in smem (as codes),
@@ -434,9 +457,235 @@ __global__ void __launch_bounds__(MergeTmaCfg<U>::kThreads) merge_tma_kernel(con
     if (tid == 0) bulk_wait_all();
 }
 
+// ---------------------------------------------------------------------------
+// Deeper pipeline (default): STAGES compact smem stages per block, each holding
+// one output tile's A range followed by its B range (na + nb = TILE keys, plus
+// alignment slack), so 3 blocks x (STAGES-1) tiles of input are in flight per
+// SM (Little's law at ~6.5 TB/s x ~1.5 us HBM / NVLink latency needs ~65 KB per
+// SM; the two-stage kernel above keeps <= 45 KB).  Every range is bulk-copied
+// from its 16-byte-aligned start to the 16-byte boundary after its end: the
+// over-fetch never leaves the 16-byte units that hold the range's own first and
+// last keys, so it cannot cross a page, and no thread-issued tail loads remain
+// on the critical path.  A stage is refilled only after the bulk store that
+// read it has finished reading (cp.async.bulk.wait_group.read).
+// ---------------------------------------------------------------------------
+struct PipeMeta {
+    int na, nb;        // keys taken from a / b
+    int offA, offB;    // smem slot of key a0 / b0 inside the stage
+};
+
+template <typename U, int STAGES_, int IPT32_ = 15>
+struct MergePipeCfg {
+    static constexpr int kStages = STAGES_;
+    static constexpr int kThreads = 256;
+    static constexpr int kIpt = sizeof(U) == 4 ? IPT32_ : (IPT32_ - 1) / 2;
+    static constexpr int kTile = kThreads * kIpt;
+    static constexpr int kV = 16 / int(sizeof(U));
+    static constexpr int kStage = (kTile + 4 * kV + kV - 1) / kV * kV;  // keys per stage
+    static constexpr size_t kSmem = size_t(kStages) * kStage * sizeof(U);
+};
+
+template <typename U, bool FLOAT, int STAGES, int IPT32>
+__global__ void __launch_bounds__(256) merge_pipe_kernel(const U* __restrict__ a, const U* __restrict__ b, uint64_t al,
+                                                         uint64_t bl, U* __restrict__ out,
+                                                         const uint64_t* __restrict__ part, uint32_t tiles) {
+    using C = MergePipeCfg<U, STAGES, IPT32>;
+    constexpr int THREADS = C::kThreads, IPT = C::kIpt, TILE = C::kTile, SK = C::kStage, V = C::kV;
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    U* stage = reinterpret_cast<U*>(smem_raw);
+    __shared__ PipeMeta meta[STAGES];
+    __shared__ __align__(8) uint64_t bar[STAGES];
+    const int tid = threadIdx.x;
+    const uint64_t total = al + bl;
+
+    auto issue = [&](uint32_t t, int s) {  // thread 0 only
+        const uint64_t k0 = uint64_t(t) * TILE;
+        const uint64_t k1 = k0 + TILE < total ? k0 + TILE : total;
+        const uint64_t a0 = part[t], a1 = part[t + 1];
+        const uint64_t b0 = k0 - a0, b1 = k1 - a1;
+        PipeMeta& m = meta[s];
+        m.na = int(a1 - a0);
+        m.nb = int(b1 - b0);
+        U* d = stage + size_t(s) * SK;
+        uint32_t bytesA = 0, bytesB = 0;
+        const void *srcA = nullptr, *srcB = nullptr;
+        int offB = 0;
+        m.offA = 0;
+        if (a1 > a0) {
+            const uintptr_t s0 = reinterpret_cast<uintptr_t>(a + a0) & ~uintptr_t(15);
+            const uintptr_t e0 = (reinterpret_cast<uintptr_t>(a + a1) + 15) & ~uintptr_t(15);
+            srcA = reinterpret_cast<const void*>(s0);
+            bytesA = uint32_t(e0 - s0);
+            m.offA = int((reinterpret_cast<uintptr_t>(a + a0) - s0) / sizeof(U));
+            offB = int(bytesA / sizeof(U));
+        }
+        m.offB = offB;
+        if (b1 > b0) {
+            const uintptr_t s0 = reinterpret_cast<uintptr_t>(b + b0) & ~uintptr_t(15);
+            const uintptr_t e0 = (reinterpret_cast<uintptr_t>(b + b1) + 15) & ~uintptr_t(15);
+            srcB = reinterpret_cast<const void*>(s0);
+            bytesB = uint32_t(e0 - s0);
+            m.offB = offB + int((reinterpret_cast<uintptr_t>(b + b0) - s0) / sizeof(U));
+        }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&bar[s])),
+                     "r"(bytesA + bytesB)
+                     : "memory");
+        if (bytesA)
+            asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                             smem_u32(d)),
+                         "l"(srcA), "r"(bytesA), "r"(smem_u32(&bar[s]))
+                         : "memory");
+        if (bytesB)
+            asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                             smem_u32(d + offB)),
+                         "l"(srcB), "r"(bytesB), "r"(smem_u32(&bar[s]))
+                         : "memory");
+    };
+    static_assert(SK >= TILE + 3 * V, "stage holds both ranges with their alignment slack");
+
+    if (tid == 0) {
+#pragma unroll
+        for (int s = 0; s < STAGES; ++s) mbar_init(&bar[s], 1);
+#pragma unroll
+        for (int s = 0; s < STAGES - 1; ++s) {
+            const uint32_t t = blockIdx.x + uint32_t(s) * gridDim.x;
+            if (t < tiles) issue(t, s);
+        }
+    }
+    __syncthreads();
+    uint32_t phases = 0;  // bit s: parity of stage s
+    int s = 0;
+    for (uint32_t t = blockIdx.x, i = 0; t < tiles; t += gridDim.x, ++i) {
+        mbar_wait(&bar[s], (phases >> s) & 1u);
+        phases ^= 1u << s;
+        const PipeMeta m = meta[s];
+        U* sbase = stage + size_t(s) * SK;
+        const U* xa = sbase + m.offA;
+        const U* xb = sbase + m.offB;
+        const int na = m.na, nb = m.nb, nt = na + nb;
+        const int d0 = min(tid * IPT, nt);
+        int lo = max(0, d0 - nb), hi = min(d0, na);
+        while (lo < hi) {
+            const int mid = (lo + hi) >> 1;
+            if (encode<U, FLOAT>(xa[mid]) <= encode<U, FLOAT>(xb[d0 - 1 - mid])) lo = mid + 1;
+            else hi = mid;
+        }
+        int ia = lo, ib = d0 - lo;
+        U r[IPT];
+        if (ia + IPT <= na && ib + IPT <= nb) {
+            // fast path (almost every thread): neither run can run out within
+            // IPT outputs, so no bounds checks; one smem load per output from
+            // an address selected by the comparison (A and B share the stage)
+            int pa = m.offA + ia, pb = m.offB + ib;
+            U va = sbase[pa], vb = sbase[pb];
+#pragma unroll
+            for (int j = 0; j < IPT; ++j) {
+                const bool takeA = encode<U, FLOAT>(va) <= encode<U, FLOAT>(vb);
+                r[j] = takeA ? va : vb;
+                pa += takeA;
+                pb += !takeA;
+                const U nx = sbase[takeA ? pa : pb];
+                va = takeA ? nx : va;
+                vb = takeA ? vb : nx;
+            }
+        } else {
+            U va = ia < na ? xa[ia] : U(0), vb = ib < nb ? xb[ib] : U(0);
+#pragma unroll
+            for (int j = 0; j < IPT; ++j) {
+                const bool takeA = ib >= nb || (ia < na && encode<U, FLOAT>(va) <= encode<U, FLOAT>(vb));
+                if (takeA) {
+                    r[j] = va;
+                    ++ia;
+                    va = ia < na ? xa[ia] : U(0);
+                } else {
+                    r[j] = vb;
+                    ++ib;
+                    vb = ib < nb ? xb[ib] : U(0);
+                }
+            }
+        }
+        __syncthreads();  // every thread is done reading this stage
+        if (d0 + IPT <= nt) {
+#pragma unroll
+            for (int j = 0; j < IPT; ++j) sbase[d0 + j] = r[j];
+        } else {
+#pragma unroll
+            for (int j = 0; j < IPT; ++j)
+                if (d0 + j < nt) sbase[d0 + j] = r[j];
+        }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        __syncthreads();
+        U* dst = out + uint64_t(t) * TILE;
+        const bool bulk = ((reinterpret_cast<uintptr_t>(dst) & 15) == 0) && ((uint32_t(nt) * sizeof(U)) % 16 == 0);
+        if (bulk) {
+            if (tid == 0) bulk_store_1d(dst, sbase, uint32_t(nt) * sizeof(U));
+        } else {
+            for (int j = tid; j < nt; j += THREADS) dst[j] = sbase[j];
+            __syncthreads();  // scalar readers done before the stage is refilled
+        }
+        // refill the stage of the previous tile (its bulk store has had a whole
+        // tile of time to drain) with the tile STAGES-1 ahead of this one
+        const int sp = s == 0 ? STAGES - 1 : s - 1;
+        const uint32_t tn = t + uint32_t(STAGES - 1) * gridDim.x;
+        if (tid == 0 && tn < tiles) {
+            asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");  // all but this tile's store
+            issue(tn, sp);
+        }
+        s = s + 1 == STAGES ? 0 : s + 1;
+        (void)i;
+        (void)V;
+    }
+    if (tid == 0) bulk_wait_all();
+}
+
+int merge_version() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = std::getenv("MSORT_MERGE_V");
+        v = e ? std::atoi(e) : 3;
+    }
+    return v;
+}
+
+template <typename U, bool FLOAT, int STAGES, int IPT32>
+cudaError_t launch_merge_pipe(const U* a, uint64_t al, const U* b, uint64_t bl, U* out, void* ws, cudaStream_t st,
+                              int* launches) {
+    using C = MergePipeCfg<U, STAGES, IPT32>;
+    constexpr uint64_t TILE = C::kTile;
+    const uint64_t tiles = (al + bl + TILE - 1) / TILE;
+    const uint64_t nparts = tiles + 1;
+    uint64_t* part = reinterpret_cast<uint64_t*>(ws);
+    partition_thread_kernel<U, FLOAT><<<unsigned((nparts + 255) / 256), 256, 0, st>>>(a, al, b, bl, TILE, nparts, part);
+    if (launches) *launches += 2;
+    auto kern = merge_pipe_kernel<U, FLOAT, STAGES, IPT32>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(C::kSmem));
+    if (e != cudaSuccess) return e;
+    int per_sm = 0, dev = 0, sms = 0;
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, C::kThreads, C::kSmem)) != cudaSuccess)
+        return e;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    uint64_t grid = uint64_t(per_sm > 0 ? per_sm : 1) * (sms > 0 ? sms : 148);
+    if (grid > tiles) grid = tiles;
+    kern<<<unsigned(grid), C::kThreads, C::kSmem, st>>>(a, b, al, bl, out, part, uint32_t(tiles));
+    return cudaGetLastError();
+}
+
 template <typename U, bool FLOAT>
 cudaError_t launch_merge_t(const void* a, uint64_t al, const void* b, uint64_t bl, void* out, void* ws,
                            cudaStream_t st, int* launches) {
+    const U *pa = (const U*)a, *pb = (const U*)b;
+    U* po = (U*)out;
+    switch (merge_version()) {
+        case 0: case 1: case 2: break;  // two-stage kernel below (round-1 reference point)
+        case 4: return launch_merge_pipe<U, FLOAT, 4, 15>(pa, al, pb, bl, po, ws, st, launches);
+        case 5: return launch_merge_pipe<U, FLOAT, 5, 15>(pa, al, pb, bl, po, ws, st, launches);
+        case 6: return launch_merge_pipe<U, FLOAT, 3, 13>(pa, al, pb, bl, po, ws, st, launches);
+        case 7: return launch_merge_pipe<U, FLOAT, 2, 15>(pa, al, pb, bl, po, ws, st, launches);
+        case 8: return launch_merge_pipe<U, FLOAT, 2, 11>(pa, al, pb, bl, po, ws, st, launches);
+        default: return launch_merge_pipe<U, FLOAT, 3, 15>(pa, al, pb, bl, po, ws, st, launches);
+    }
     using C = MergeTmaCfg<U>;
     constexpr uint64_t TILE = C::kTile;
     const uint64_t total = al + bl;
@@ -518,8 +767,9 @@ cudaError_t launch_splitters(const GroupPtrs& all, int g, uint64_t c, int kt, ui
 }
 
 size_t merge_ws_bytes(uint64_t total, int kt) {
-    const uint64_t tile = key_bytes(kt) == 4 ? uint64_t(MergeCfg<uint32_t>::kThreads) * MergeCfg<uint32_t>::kIpt
-                                             : uint64_t(MergeCfg<uint64_t>::kThreads) * MergeCfg<uint64_t>::kIpt;
+    // smallest tile of any merge configuration (MergePipeCfg<.., 11> for the tuning variants)
+    const uint64_t tile = key_bytes(kt) == 4 ? uint64_t(MergePipeCfg<uint32_t, 2, 11>::kTile)
+                                             : uint64_t(MergePipeCfg<uint64_t, 2, 11>::kTile);
     return size_t((total + tile - 1) / tile + 2) * 8 + 256;
 }
 

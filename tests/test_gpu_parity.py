@@ -189,6 +189,29 @@ def test_step_merge(ms, kt):
         assert np.array_equal(bits(got, kt), bits(expect, kt)), (al, bl)
 
 
+@pytest.mark.parametrize("kt", ["u32", "u64"])
+def test_step_merge_unaligned(ms, kt):
+    """Runs and output starting at any key offset (the merge bulk-copies each
+    range from its 16-byte-aligned start to the 16-byte boundary after its end;
+    the ragged output goes through the scalar store path)."""
+    K = mi.KEY_BYTES[kt]
+    for (oa, ob, oo), (al, bl) in [((1, 2, 0), (40000, 33333)), ((3, 0, 1), (3841, 7681)), ((2, 3, 3), (5, 100001)),
+                                    ((1, 1, 2), (65536, 65536)), ((0, 1, 0), (1, 123457))]:
+        a = sort.oracle_sort(mi.np_generate(al, kt, "uniform", seed=oa + 11), kt)
+        b = sort.oracle_sort(mi.np_generate(bl, kt, "uniform", seed=ob + 13), kt)
+        da = dev_keys(np.concatenate([np.zeros(oa, a.dtype), a]))
+        db = dev_keys(np.concatenate([np.zeros(ob, b.dtype), b]))
+        out = torch.zeros((al + bl + oo) * K, dtype=torch.uint8, device="cuda")
+        wsb = ms.msort_merge_workspace_bytes(al + bl, kt)
+        ws = torch.empty(wsb, dtype=torch.uint8, device="cuda")
+        ms.msort_step_merge(ms.tensor_ptr(da) + oa * K, al, ms.tensor_ptr(db) + ob * K, bl, ms.tensor_ptr(out) + oo * K,
+                            kt, ms.tensor_ptr(ws), wsb)
+        torch.cuda.synchronize()
+        got = host_keys(out, kt)[oo: oo + al + bl]
+        expect = sort.oracle_sort(np.concatenate([a, b]), kt)
+        assert np.array_equal(bits(got, kt), bits(expect, kt)), (oa, ob, oo, al, bl)
+
+
 def _virtual_sort(ms, a, kt, g, exchange=0):
     """g virtual ranks on GPU 0, device-resident chunks of c keys."""
     n = len(a)

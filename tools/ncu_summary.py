@@ -26,3 +26,8 @@ print("stall samples", tot)
 n = int(sys.argv[2]) if len(sys.argv) > 2 else 25
 for x in sorted(data, key=lambda x: -int(x[i_s]) if x[i_s].isdigit() else 0)[:n]:
     print(f"{int(x[i_s]):7d} {x[0][-5:]} {x[1][:100]}")
+# warp-state breakdown (cycles per issued instruction by stall reason)
+st = [(hdr[i], vals[i]) for i in range(len(hdr)) if hdr[i].startswith('smsp__average_warps_issue_stalled_')
+      and hdr[i].endswith('_per_issue_active.ratio')]
+st = sorted(((float(v.replace(',', '')) if v.replace(',', '').replace('.', '').isdigit() else 0.0, k) for k, v in st), reverse=True)
+print("warp stalls (per issue):", ", ".join(f"{k[len('smsp__average_warps_issue_stalled_'):-len('_per_issue_active.ratio')]}={v:.2f}" for v, k in st[:8]))
