@@ -498,10 +498,11 @@ __global__ void __launch_bounds__(256) merge_pipe_kernel(const U* __restrict__ a
     const int tid = threadIdx.x;
     const uint64_t total = al + bl;
 
-    auto issue = [&](uint32_t t, int s) {  // thread 0 only
+    // thread 0 only; a0/a1 = part[t], part[t+1] (loaded one tile ahead, so the
+    // refill never waits on a global load while the other warps wait for it)
+    auto issue = [&](uint32_t t, int s, uint64_t a0, uint64_t a1) {
         const uint64_t k0 = uint64_t(t) * TILE;
         const uint64_t k1 = k0 + TILE < total ? k0 + TILE : total;
-        const uint64_t a0 = part[t], a1 = part[t + 1];
         const uint64_t b0 = k0 - a0, b1 = k1 - a1;
         PipeMeta& m = meta[s];
         m.na = int(a1 - a0);
@@ -550,13 +551,19 @@ __global__ void __launch_bounds__(256) merge_pipe_kernel(const U* __restrict__ a
 #pragma unroll
         for (int s = 0; s < STAGES - 1; ++s) {
             const uint32_t t = blockIdx.x + uint32_t(s) * gridDim.x;
-            if (t < tiles) issue(t, s);
+            if (t < tiles) issue(t, s, part[t], part[t + 1]);
         }
     }
     __syncthreads();
     uint32_t phases = 0;  // bit s: parity of stage s
     int s = 0;
     for (uint32_t t = blockIdx.x, i = 0; t < tiles; t += gridDim.x, ++i) {
+        const uint32_t tn = t + uint32_t(STAGES - 1) * gridDim.x;
+        uint64_t pa0 = 0, pa1 = 0;
+        if (tid == 0 && tn < tiles) {
+            pa0 = __ldg(part + tn);
+            pa1 = __ldg(part + tn + 1);
+        }
         mbar_wait(&bar[s], (phases >> s) & 1u);
         phases ^= 1u << s;
         const PipeMeta m = meta[s];
@@ -573,12 +580,15 @@ __global__ void __launch_bounds__(256) merge_pipe_kernel(const U* __restrict__ a
         }
         int ia = lo, ib = d0 - lo;
         U r[IPT];
-        if (ia + IPT <= na && ib + IPT <= nb) {
-            // fast path (almost every thread): neither run can run out within
-            // IPT outputs, so no bounds checks; one smem load per output from
-            // an address selected by the comparison (A and B share the stage)
-            int pa = m.offA + ia, pb = m.offB + ib;
-            U va = sbase[pa], vb = sbase[pb];
+        // One smem load per output from an address selected by the comparison
+        // (A and B share the stage; a read one past the end of a run stays in
+        // the stage and is never used).  The path is chosen per WARP: a warp
+        // whose lanes cannot exhaust a run within IPT outputs (almost all)
+        // skips the bounds predicates; otherwise every lane runs the predicated
+        // loop, so no warp executes both paths.
+        int pa = m.offA + ia, pb = m.offB + ib;
+        U va = sbase[pa], vb = sbase[pb];
+        if (__all_sync(0xffffffffu, ia + IPT <= na && ib + IPT <= nb)) {
 #pragma unroll
             for (int j = 0; j < IPT; ++j) {
                 const bool takeA = encode<U, FLOAT>(va) <= encode<U, FLOAT>(vb);
@@ -590,19 +600,16 @@ __global__ void __launch_bounds__(256) merge_pipe_kernel(const U* __restrict__ a
                 vb = takeA ? vb : nx;
             }
         } else {
-            U va = ia < na ? xa[ia] : U(0), vb = ib < nb ? xb[ib] : U(0);
+            const int ea = m.offA + na, eb = m.offB + nb;  // one past the end of each run
 #pragma unroll
             for (int j = 0; j < IPT; ++j) {
-                const bool takeA = ib >= nb || (ia < na && encode<U, FLOAT>(va) <= encode<U, FLOAT>(vb));
-                if (takeA) {
-                    r[j] = va;
-                    ++ia;
-                    va = ia < na ? xa[ia] : U(0);
-                } else {
-                    r[j] = vb;
-                    ++ib;
-                    vb = ib < nb ? xb[ib] : U(0);
-                }
+                const bool takeA = pb >= eb || (pa < ea && encode<U, FLOAT>(va) <= encode<U, FLOAT>(vb));
+                r[j] = takeA ? va : vb;
+                pa += takeA;
+                pb += !takeA;
+                const U nx = sbase[takeA ? pa : pb];
+                va = takeA ? nx : va;
+                vb = takeA ? vb : nx;
             }
         }
         __syncthreads();  // every thread is done reading this stage
@@ -627,10 +634,9 @@ __global__ void __launch_bounds__(256) merge_pipe_kernel(const U* __restrict__ a
         // refill the stage of the previous tile (its bulk store has had a whole
         // tile of time to drain) with the tile STAGES-1 ahead of this one
         const int sp = s == 0 ? STAGES - 1 : s - 1;
-        const uint32_t tn = t + uint32_t(STAGES - 1) * gridDim.x;
         if (tid == 0 && tn < tiles) {
             asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");  // all but this tile's store
-            issue(tn, sp);
+            issue(tn, sp, pa0, pa1);
         }
         s = s + 1 == STAGES ? 0 : s + 1;
         (void)i;
