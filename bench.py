@@ -59,7 +59,7 @@ def parse():
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--exchange", type=int, default=0,
                     help="merge phase for N>1: 0 the paper's Alg.2 with fused exchange+merge, 1 Alg.2 swap then "
-                         "merge (single process only), 2 NEXT-1 single all-to-all")
+                         "merge (single process only), 2 NEXT-1 single all-to-all fused into the merge, 3 NEXT-1 pull then merge")
     ap.add_argument("--het", action="store_true", help="also time the HET-sort baseline (GPU chunk sort + CPU merge)")
     ap.add_argument("--het-chunks", type=int, default=8)
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -394,7 +394,7 @@ def main():
                        "n": n, "keys_per_gpu": c, "key_type": kt, "distribution": args.dist, "seed": args.seed,
                        "parallelism": f"p2p{g}", "l2": "inputs 16 GB >> 126 MB L2 (no flush needed)",
                        "exchange": ["Alg.2, fused peer-read merge", "Alg.2, swap then merge",
-                                    "NEXT-1 single all-to-all"][args.exchange] if g > 1 else "none (1 GPU)"},
+                                    "NEXT-1 single all-to-all fused into the merge", "NEXT-1 single all-to-all, pull then merge"][args.exchange] if g > 1 else "none (1 GPU)"},
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
             "clocks": clk.summary(), "wall_s_timed_region": wall,
             "step_ms": {"min": min(step_ms), "max": max(step_ms)},

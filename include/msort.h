@@ -111,8 +111,11 @@ enum {
                                        NVLink directly (default); 1: swap first (peer copy into a receive
                                        buffer), then a local merge;
                                        2: NEXT-1, the paper's future work: exact multi-sequence
-                                       splitters over all g sorted chunks, ONE all-to-all exchange (every GPU
-                                       pulls its run from every chunk), local log2(g)-round merge tree       */
+                                       splitters over all g sorted chunks, ONE all-to-all exchange fused into
+                                       a log2(g)-round merge tree whose first round reads the g runs straight
+                                       from the peers' chunks over NVLink;
+                                       3: NEXT-1 with the exchange as separate pulls (every GPU copies its run
+                                       from every chunk into a local buffer), then the merge tree            */
     MSORT_OPT_SKIP_TRIVIAL = 2   /* 1: skip radix passes whose digit is constant (identity permutation)   */
 };
 int msort_set_option(msort_ctx* ctx, int option, int64_t value);

@@ -29,7 +29,7 @@ MSORT_MAX_GPUS = 8
 MSORT_MAX_STAGES = 7
 MSORT_DIST_HANDLE_BYTES = 512
 MSORT_OPT_TIMING, MSORT_OPT_EXCHANGE, MSORT_OPT_SKIP_TRIVIAL = 0, 1, 2
-EXCHANGE_FUSED, EXCHANGE_SWAP, EXCHANGE_ALLTOALL = 0, 1, 2
+EXCHANGE_FUSED, EXCHANGE_SWAP, EXCHANGE_ALLTOALL, EXCHANGE_ALLTOALL_PULL = 0, 1, 2, 3
 MSORT_PASS_ENCODE_IN, MSORT_PASS_DECODE_OUT = 1, 2
 
 STATUS = {0: "MSORT_OK", 1: "MSORT_ERR_INVALID_ARGUMENT", 2: "MSORT_ERR_DEVICE", 3: "MSORT_ERR_OUT_OF_MEMORY",

@@ -22,7 +22,10 @@ struct RadixWs {
     uint64_t tiles;
     uint64_t groups;
     size_t head_bytes;            // bytes of counters..trivial
-    size_t zero_bytes;            // head + status words + group aggregates: zeroed once per sort
+    size_t zero_bytes;            // head + status words + group aggregates
+    uint32_t epoch = 0;           // 0: zero the whole workspace and tag status words pass+1; else only the
+                                  // head and the group aggregates are zeroed and status words carry
+                                  // (epoch << 4 | pass+1), so words of earlier sorts never match
 };
 uint32_t radix_tile_keys(int kt);
 size_t radix_ws_bytes(uint64_t n, int kt);

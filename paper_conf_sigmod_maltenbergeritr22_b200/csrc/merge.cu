@@ -649,7 +649,7 @@ int merge_version() {
     static int v = -1;
     if (v < 0) {
         const char* e = std::getenv("MSORT_MERGE_V");
-        v = e ? std::atoi(e) : 3;
+        v = e ? std::atoi(e) : 12;  // 12 = the per-key-type default below
     }
     return v;
 }
@@ -690,7 +690,13 @@ cudaError_t launch_merge_t(const void* a, uint64_t al, const void* b, uint64_t b
         case 6: return launch_merge_pipe<U, FLOAT, 3, 13>(pa, al, pb, bl, po, ws, st, launches);
         case 7: return launch_merge_pipe<U, FLOAT, 2, 15>(pa, al, pb, bl, po, ws, st, launches);
         case 8: return launch_merge_pipe<U, FLOAT, 2, 11>(pa, al, pb, bl, po, ws, st, launches);
-        default: return launch_merge_pipe<U, FLOAT, 3, 15>(pa, al, pb, bl, po, ws, st, launches);
+        case 9: return launch_merge_pipe<U, FLOAT, 3, 23>(pa, al, pb, bl, po, ws, st, launches);
+        case 10: return launch_merge_pipe<U, FLOAT, 2, 31>(pa, al, pb, bl, po, ws, st, launches);
+        case 11: return launch_merge_pipe<U, FLOAT, 3, 19>(pa, al, pb, bl, po, ws, st, launches);
+        case 3: return launch_merge_pipe<U, FLOAT, 3, 15>(pa, al, pb, bl, po, ws, st, launches);
+        default:  // measured best (profiles/merge_tuning_r1.md): 3 stages, 19 keys/thread (u32), 11 (u64)
+            if constexpr (sizeof(U) == 4) return launch_merge_pipe<U, FLOAT, 3, 19>(pa, al, pb, bl, po, ws, st, launches);
+            else return launch_merge_pipe<U, FLOAT, 3, 23>(pa, al, pb, bl, po, ws, st, launches);
     }
     using C = MergeTmaCfg<U>;
     constexpr uint64_t TILE = C::kTile;

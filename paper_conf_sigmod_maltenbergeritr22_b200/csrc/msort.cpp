@@ -150,6 +150,9 @@ struct Rank {
     int cur = -1;  // -1: user buffer, 0..2: buf[]
     int passes_run = 0;
     int pass_ids[8] = {};
+    // radix workspace epoch (RadixWs::epoch); starts so that the first sort
+    // zeroes the whole workspace, and wraps to 0 (full zeroing) every 2^26 sorts
+    uint32_t radix_epoch = (1u << 26) - 1;
 
     void* ptr(int which) const { return which < 0 ? user : buf[which]; }
 };
@@ -264,6 +267,8 @@ float elapsed(cudaEvent_t a, cudaEvent_t b) {
 int radix_begin(msort_ctx* ctx, Rank& R, const void* src, uint64_t c) {
     CUDA_TRY(cudaSetDevice(R.dev));
     RadixWs ws = radix_ws_layout(R.rws, c, ctx->kt);
+    R.radix_epoch = (R.radix_epoch + 1) & ((1u << 26) - 1);
+    ws.epoch = R.radix_epoch;
     CUDA_TRY(radix_prologue(src, c, ctx->kt, ws, R.st));
     ctx->tm.kernel_launches += 2;
     if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_hist, R.st));
@@ -277,6 +282,7 @@ int radix_passes(msort_ctx* ctx, Rank& R, const void* src, void* dst, void* tmp,
     CUDA_TRY(cudaSetDevice(R.dev));
     const int P = num_passes(ctx->kt);
     RadixWs ws = radix_ws_layout(R.rws, c, ctx->kt);
+    ws.epoch = R.radix_epoch;
     bool run[8];
     int nrun = 0;
     for (int p = 0; p < P; ++p) {
@@ -440,6 +446,45 @@ int merge_tree(msort_ctx* ctx, Rank& R, const Runs& runs, int g, char* src, char
     return MSORT_OK;
 }
 
+// NEXT-1 fused (exchange mode 2): the first round of the merge tree reads the
+// g runs straight from the peers' sorted chunks (B1) over NVLink, so pulled keys
+// never make an HBM round trip.  Rounds alternate between d_user and B0 so that
+// the last one lands in d_user and no round writes B1, which peers may still be
+// reading (the caller orders the next use of B1 after every rank's merges).
+int merge_tree_from_peers(msort_ctx* ctx, Rank& R, const Runs& runs, const char* const* run_ptr, int g, char* buf0,
+                          char* d_user, bool time_first_round) {
+    const size_t K = key_bytes(ctx->kt);
+    int levels = 0;
+    while ((1 << levels) < g) ++levels;
+    uint64_t off[MSORT_MAX_GPUS], len[MSORT_MAX_GPUS];
+    for (int r = 0; r < g; ++r) {
+        off[r] = runs.off[r];
+        len[r] = runs.len[r];
+    }
+    char* in = nullptr;
+    for (int lv = 1, nr = g; lv <= levels; ++lv) {
+        char* o = ((levels - lv) % 2 == 0) ? d_user : buf0;
+        if (lv == 1 && time_first_round) CUDA_TRY(cudaEventRecord(R.e_xch[0][0], R.st));
+        int m = 0;
+        for (int i = 0; i + 1 < nr; i += 2) {
+            const char* a = lv == 1 ? run_ptr[i] : in + off[i] * K;
+            const char* b = lv == 1 ? run_ptr[i + 1] : in + off[i + 1] * K;
+            CUDA_TRY(launch_merge(a, len[i], b, len[i + 1], o + off[i] * K, ctx->kt, R.mws, R.st,
+                                  &ctx->tm.kernel_launches));
+            off[m] = off[i];
+            len[m] = len[i] + len[i + 1];
+            ++m;
+        }
+        if (lv == 1 && time_first_round) {
+            CUDA_TRY(cudaEventRecord(R.e_xch[0][1], R.st));
+            R.xch_rec[0] = true;
+        }
+        nr = m;
+        in = o;
+    }
+    return MSORT_OK;
+}
+
 int alltoall_local(msort_ctx* ctx, uint64_t c) {
     const int g = ctx->g;
     const size_t K = key_bytes(ctx->kt);
@@ -466,6 +511,30 @@ int alltoall_local(msort_ctx* ctx, uint64_t c) {
     CUDA_TRY(cudaStreamSynchronize(R0.st));
     std::vector<uint64_t> s(R0.h_pivot, R0.h_pivot + (g + 1) * g);
     record_alltoall_stats(ctx, s.data(), g);
+    if (ctx->exchange == 2) {
+        // fused: every rank merges its runs straight out of the peers' B1
+        for (int j = 0; j < g; ++j) {
+            Rank& R = ctx->r[j];
+            CUDA_TRY(cudaSetDevice(R.dev));
+            const Runs rr = runs_of(s.data(), g, j);
+            const char* rp[MSORT_MAX_GPUS];
+            for (int r = 0; r < g; ++r) rp[r] = static_cast<const char*>(ctx->r[r].buf[1]) + s[j * g + r] * K;
+            MSORT_TRY(merge_tree_from_peers(ctx, R, rr, rp, g, static_cast<char*>(R.buf[0]),
+                                            static_cast<char*>(R.user), ctx->timing != 0));
+            if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[0][1], R.st));
+            CUDA_TRY(cudaEventRecord(R.e_sync[1], R.st));
+        }
+        // no rank's B1 is reused (next sort) before every rank finished reading it
+        for (int j = 0; j < g; ++j) {
+            Rank& R = ctx->r[j];
+            CUDA_TRY(cudaSetDevice(R.dev));
+            for (int q = 0; q < g; ++q)
+                if (q != j) CUDA_TRY(cudaStreamWaitEvent(R.st, ctx->r[q].e_sync[1], 0));
+            R.cur = -1;
+            CUDA_TRY(cudaEventRecord(R.e_end, R.st));
+        }
+        return MSORT_OK;
+    }
     // the single exchange: rank j pulls its run from every chunk into B0
     for (int j = 0; j < g; ++j) {
         Rank& R = ctx->r[j];
@@ -520,7 +589,7 @@ int sort_device_local(msort_ctx* ctx, uint64_t c) {
         }
         CUDA_TRY(cudaEventRecord(R.e_sorted, R.st));
     }
-    if (g > 1 && ctx->exchange == 2) return alltoall_local(ctx, c);
+    if (g > 1 && ctx->exchange >= 2) return alltoall_local(ctx, c);
     const int S = int(labels.size());
     ctx->tm.n_stages = S;
     for (int s = 0; s < S; ++s) {
@@ -833,7 +902,7 @@ int msort_set_option(msort_ctx* ctx, int option, int64_t value) {
         case MSORT_OPT_TIMING: ctx->timing = value ? 1 : 0; return MSORT_OK;
         case MSORT_OPT_SKIP_TRIVIAL: ctx->skip_trivial = value ? 1 : 0; return MSORT_OK;
         case MSORT_OPT_EXCHANGE:
-            if (value < 0 || value > 2) return set_error(MSORT_ERR_INVALID_ARGUMENT, "exchange mode 0, 1 or 2");
+            if (value < 0 || value > 3) return set_error(MSORT_ERR_INVALID_ARGUMENT, "exchange mode 0, 1, 2 or 3");
             if (value == 1)
                 for (int i = 0; i < ctx->nlocal; ++i)
                     if (!ctx->r[i].buf[2]) {
@@ -1193,7 +1262,7 @@ static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* strea
         for (int q = 0; q < g; ++q) cur[q] = 1;
     }
     CUDA_TRY(cudaEventRecord(R.e_sorted, R.st));
-    if (g > 1 && ctx->exchange == 2) {
+    if (g > 1 && ctx->exchange >= 2) {
         // NEXT-1: splitters from every peer's sorted chunk, one pull per peer,
         // barrier (peers' B1 no longer read), local merge tree into d_chunk
         const size_t K = key_bytes(ctx->kt);
@@ -1211,18 +1280,29 @@ static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* strea
         std::vector<uint64_t> s(R.h_pivot, R.h_pivot + (g + 1) * g);
         record_alltoall_stats(ctx, s.data(), g);
         const Runs rr = runs_of(s.data(), g, me);
-        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[0][0], R.st));
-        for (int q = 0; q < g; ++q)
-            if (rr.len[q])
-                CUDA_TRY(cudaMemcpyAsync(static_cast<char*>(R.buf[0]) + rr.off[q] * K,
-                                         static_cast<const char*>(ctx->peer_buf[q][1]) + s[me * g + q] * K, rr.len[q] * K,
-                                         cudaMemcpyDefault, R.st));
-        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[0][1], R.st));
-        R.xch_rec[0] = ctx->timing != 0;
-        MSORT_TRY(dist_barrier(ctx));  // every rank finished pulling from our B1
-        MSORT_TRY(merge_tree(ctx, R, rr, g, static_cast<char*>(R.buf[0]), static_cast<char*>(R.buf[1]),
-                             static_cast<char*>(d_chunk)));
-        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[0][1], R.st));
+        if (ctx->exchange == 2) {
+            // fused: merge straight out of the peers' B1, then one barrier so that
+            // no rank reuses its B1 while a peer may still be reading it
+            const char* rp[MSORT_MAX_GPUS];
+            for (int q = 0; q < g; ++q) rp[q] = static_cast<const char*>(ctx->peer_buf[q][1]) + s[me * g + q] * K;
+            MSORT_TRY(merge_tree_from_peers(ctx, R, rr, rp, g, static_cast<char*>(R.buf[0]),
+                                            static_cast<char*>(d_chunk), ctx->timing != 0));
+            if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[0][1], R.st));
+            MSORT_TRY(dist_barrier(ctx));
+        } else {
+            if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[0][0], R.st));
+            for (int q = 0; q < g; ++q)
+                if (rr.len[q])
+                    CUDA_TRY(cudaMemcpyAsync(static_cast<char*>(R.buf[0]) + rr.off[q] * K,
+                                             static_cast<const char*>(ctx->peer_buf[q][1]) + s[me * g + q] * K, rr.len[q] * K,
+                                             cudaMemcpyDefault, R.st));
+            if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[0][1], R.st));
+            R.xch_rec[0] = ctx->timing != 0;
+            MSORT_TRY(dist_barrier(ctx));  // every rank finished pulling from our B1
+            MSORT_TRY(merge_tree(ctx, R, rr, g, static_cast<char*>(R.buf[0]), static_cast<char*>(R.buf[1]),
+                                 static_cast<char*>(d_chunk)));
+            if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[0][1], R.st));
+        }
         CUDA_TRY(cudaEventRecord(R.e_end, R.st));
         CUDA_TRY(cudaMemcpyAsync(R.h_err, R.d_err, sizeof(int), cudaMemcpyDeviceToHost, R.st));
         CUDA_TRY(cudaStreamWaitEvent(ust, R.e_end, 0));

@@ -554,12 +554,14 @@ using Cfg32_4 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 32>;  // lo
 using Cfg32_5 = OsCfg<256, 28, 0x5555555u, 4, true, 6, false, false, 32>;  // window 6, groups of 32
 using Cfg32_6 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, true>;       // count atomic's return = rank
 using Cfg32_7 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 8>;   // window 4, groups of 8
+using Cfg32_8 = OsCfg<256, 24, 0x555555u, 5, true, 2, false, false, 32>;   // 6144-key tiles, 5 blocks/SM (40 warps)
+using Cfg32_9 = OsCfg<256, 20, 0x55555u, 6, true, 2, false, false, 32>;    // 5120-key tiles, 6 blocks/SM (48 warps)
 using Cfg64_0 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 16>;     // prefetch, groups of 16 (best)
 using Cfg64_1 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 0>;      // tile-by-tile look-back only
 using Cfg64_2 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 8>;      // groups of 8
 using Cfg64_3 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 32>;     // groups of 32
 
-constexpr uint32_t kMinTile32 = 256 * 28;  // smallest u32 tile above
+constexpr uint32_t kMinTile32 = 256 * 20;  // smallest u32 tile above (sizes the status array)
 constexpr uint32_t kMinTile64 = 256 * 14;  // smallest u64 tile above
 
 int env_cfg() {
@@ -567,7 +569,7 @@ int env_cfg() {
     if (v < 0) {
         const char* e = std::getenv("MSORT_OS_CFG");
         v = e ? std::atoi(e) : 0;
-        if (v < 0 || v > 7) v = 0;
+        if (v < 0 || v > 9) v = 0;
     }
     return v;
 }
@@ -666,6 +668,8 @@ cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, c
             case 5: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_5, STABLE>(in, out, n, pass, ws, base_row, tag, st);
             case 6: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_6, STABLE>(in, out, n, pass, ws, base_row, tag, st);
             case 7: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_7, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            case 8: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_8, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            case 9: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_9, STABLE>(in, out, n, pass, ws, base_row, tag, st);
             default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_0, STABLE>(in, out, n, pass, ws, base_row, tag, st);
         }
     } else {
@@ -673,7 +677,7 @@ cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, c
             case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_1, STABLE>(in, out, n, pass, ws, base_row, tag, st);
             case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_2, STABLE>(in, out, n, pass, ws, base_row, tag, st);
             case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_3, STABLE>(in, out, n, pass, ws, base_row, tag, st);
-            case 4: case 5: case 6: case 7:
+            case 4: case 5: case 6: case 7: case 8: case 9:
                 return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st);
             default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st);
         }
@@ -723,7 +727,22 @@ static size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
 static size_t head_bytes() { return align_up(8 * 4 + 8 * 256 * 4 * 2 + 16 * 4, 256); }
 
-constexpr uint64_t kMinGroup = 8;  // smallest look-back group of the configs above
+constexpr uint64_t kMinGroup = 8;  // smallest look-back group of the configs above (sizes the allocation)
+
+// look-back group size of the configuration in use (gagg stride; only that much is zeroed per sort)
+static uint64_t active_group(int kt) {
+    const int c = env_cfg();
+    uint32_t gsz;
+    if (key_bytes(kt) == 4) {
+        constexpr uint32_t G32[10] = {Cfg32_0::kGroup, Cfg32_1::kGroup, Cfg32_2::kGroup, Cfg32_3::kGroup, Cfg32_4::kGroup,
+                                      Cfg32_5::kGroup, Cfg32_6::kGroup, Cfg32_7::kGroup, Cfg32_8::kGroup, Cfg32_9::kGroup};
+        gsz = G32[c];
+    } else {
+        constexpr uint32_t G64[4] = {Cfg64_0::kGroup, Cfg64_1::kGroup, Cfg64_2::kGroup, Cfg64_3::kGroup};
+        gsz = G64[c < 4 ? c : 0];
+    }
+    return gsz ? gsz : kMinGroup;
+}
 
 static uint64_t ws_groups(uint64_t tiles) { return tiles / kMinGroup + 1; }
 
@@ -743,7 +762,7 @@ RadixWs radix_ws_layout(void* ws, uint64_t n, int kt) {
     w.head_bytes = head_bytes();
     w.status = reinterpret_cast<unsigned long long*>(p + w.head_bytes);
     w.tiles = (n + radix_tile_keys(kt) - 1) / radix_tile_keys(kt);
-    w.groups = ws_groups(w.tiles);
+    w.groups = w.tiles / active_group(kt) + 1;  // <= ws_groups(tiles): the allocation covers any config
     w.gagg = reinterpret_cast<unsigned long long*>(p + w.head_bytes + align_up(size_t(w.tiles) * kRadix * 8, 256));
     w.zero_bytes = w.head_bytes + align_up(size_t(w.tiles) * kRadix * 8, 256) +
                    size_t(num_passes(kt)) * w.groups * kRadix * 8;
@@ -783,7 +802,16 @@ cudaError_t launch_scan(const uint32_t* hist, uint32_t* base, uint32_t* trivial,
 }
 
 cudaError_t radix_prologue(const void* keys, uint64_t n, int kt, const RadixWs& ws, cudaStream_t st) {
-    cudaError_t e = cudaMemsetAsync(ws.counters, 0, ws.zero_bytes, st);
+    cudaError_t e;
+    if (ws.epoch == 0) {
+        e = cudaMemsetAsync(ws.counters, 0, ws.zero_bytes, st);
+    } else {
+        // epoch-tagged status words need no zeroing (1.1 GB at 4e9 keys); the
+        // per-pass tile counters and the group aggregates (atomic sums) do
+        e = cudaMemsetAsync(ws.counters, 0, ws.head_bytes, st);
+        if (e == cudaSuccess)
+            e = cudaMemsetAsync(ws.gagg, 0, size_t(num_passes(kt)) * ws.groups * kRadix * 8, st);
+    }
     if (e != cudaSuccess) return e;
     if ((e = launch_histogram(keys, n, kt, ws.hist, st)) != cudaSuccess) return e;
     return launch_scan(ws.hist, ws.base, ws.trivial, n, kt, st);
@@ -792,7 +820,8 @@ cudaError_t radix_prologue(const void* keys, uint64_t n, int kt, const RadixWs& 
 cudaError_t launch_onesweep(const void* in, void* out, uint64_t n, int kt, int pass, int flags, const RadixWs& ws,
                             const uint32_t* base_row, cudaStream_t st) {
     if (n == 0) return cudaSuccess;
-    const uint32_t tag = uint32_t(pass) + 1;  // status words of other passes are ignored
+    // status words of other passes and of earlier sorts (epochs) are ignored
+    const uint32_t tag = ((ws.epoch << 4) + uint32_t(pass) + 1) & 0x3FFFFFFFu;
     switch (kt) {
         case 0: return launch_onesweep_int<uint32_t>(in, out, n, pass, flags, ws, base_row, tag, st);
         case 1: return launch_onesweep_int<uint64_t>(in, out, n, pass, flags, ws, base_row, tag, st);

@@ -53,6 +53,24 @@ def test_radix_sort_single_gpu(ms, kt, n):
     assert np.array_equal(bits(host_keys(d, kt), kt), bits(sort.oracle_sort(a, kt), kt))
 
 
+@pytest.mark.parametrize("g", [1, 4])
+def test_repeated_sorts_one_context(ms, g):
+    """Look-back status words are not zeroed between sorts of one context (they
+    carry a per-sort epoch tag): back-to-back sorts of different sizes and
+    inputs in one context must each match the oracle."""
+    cap = 4 * 60000
+    ctx = ms.Context(g, cap, "u32", device_ids=[0] * g)
+    for i, n in enumerate([cap, 4 * 7000, cap, 4 * 123, cap - 4 * 999, cap]):
+        c = n // g
+        a = mi.np_generate(g * c, "u32", ["uniform", "zipf", "reverse"][i % 3], seed=100 + i)
+        chunks = [dev_keys(a[j * c:(j + 1) * c]) for j in range(g)]
+        ctx.sort_device([ms.tensor_ptr(t) for t in chunks], c)
+        torch.cuda.synchronize()
+        got = np.concatenate([host_keys(t, "u32") for t in chunks])
+        assert np.array_equal(got, sort.oracle_sort(a, "u32")), (i, n)
+    ctx.close()
+
+
 @pytest.mark.parametrize("dist", mi.DISTRIBUTIONS)
 def test_radix_sort_distributions(ms, dist):
     n = 3 * (1 << 18) + 77
@@ -289,7 +307,7 @@ def test_errors(ms):
 
 
 # ---------------------------------------------------------------------------
-# NEXT-1: single all-to-all exchange (MSORT_OPT_EXCHANGE = 2)
+# NEXT-1: single all-to-all exchange (MSORT_OPT_EXCHANGE = 2 fused, 3 pull-then-merge)
 # ---------------------------------------------------------------------------
 
 @pytest.mark.parametrize("g", [2, 4, 8])
@@ -312,21 +330,23 @@ def test_step_splitters(ms, g):
         assert got == expect, (kt, c)
 
 
+@pytest.mark.parametrize("exchange", [2, 3])  # 2: pulls fused into the first merge round, 3: pull, then merge
 @pytest.mark.parametrize("g", [2, 4, 8])
 @pytest.mark.parametrize("dist", ["uniform", "sorted", "reverse", "zipf", "zipf_rank"])
-def test_alltoall_virtual_ranks(ms, g, dist):
+def test_alltoall_virtual_ranks(ms, g, dist, exchange):
     c = 3 * 7168 + 52
     a = mi.np_generate(g * c, "u32", dist, seed=g + 7)
-    out, tm = _virtual_sort(ms, a, "u32", g, exchange=2)
+    out, tm = _virtual_sort(ms, a, "u32", g, exchange=exchange)
     assert np.array_equal(out, sort.oracle_sort(a, "u32"))
     assert tm["n_stages"] == 1 and tm["stage_label"] == [g]
 
 
+@pytest.mark.parametrize("exchange", [2, 3])
 @pytest.mark.parametrize("kt", ["u64", "f32", "f64"])
-def test_alltoall_virtual_key_types(ms, kt):
+def test_alltoall_virtual_key_types(ms, kt, exchange):
     g, c = 8, 4001
     a = mi.np_generate(g * c, kt, "uniform", seed=33)
-    out, _ = _virtual_sort(ms, a, kt, g, exchange=2)
+    out, _ = _virtual_sort(ms, a, kt, g, exchange=exchange)
     assert np.array_equal(bits(out, kt), bits(sort.oracle_sort(a, kt), kt))
 
 
