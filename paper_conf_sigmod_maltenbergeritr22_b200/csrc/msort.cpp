@@ -135,7 +135,7 @@ struct Rank {
     size_t mws_bytes = 0;
     uint64_t* d_pivot = nullptr;   // [128] pivots (Alg.2) or splitters (all-to-all)
     uint64_t* h_pivot = nullptr;   // pinned [128]
-    uint32_t* h_trivial = nullptr; // pinned [16]: trivial flags, largest bin per pass
+    uint32_t* h_trivial = nullptr; // pinned [24]: trivial flags, largest bin per pass, its digit
     int* d_err = nullptr;          // barrier timeout flag
     int* h_err = nullptr;          // pinned
     cudaEvent_t e_begin = nullptr, e_hist = nullptr, e_sorted = nullptr, e_end = nullptr;
@@ -206,7 +206,7 @@ int alloc_rank(msort_ctx* ctx, Rank& R, bool need_b1, bool need_stage) {
     CUDA_TRY(cudaMalloc(&R.d_err, sizeof(int)));
     CUDA_TRY(cudaMemset(R.d_err, 0, sizeof(int)));
     CUDA_TRY(cudaMallocHost(&R.h_pivot, 128 * sizeof(uint64_t)));
-    CUDA_TRY(cudaMallocHost(&R.h_trivial, 16 * sizeof(uint32_t)));
+    CUDA_TRY(cudaMallocHost(&R.h_trivial, 24 * sizeof(uint32_t)));
     CUDA_TRY(cudaMallocHost(&R.h_err, sizeof(int)));
     *R.h_err = 0;
     cudaEvent_t* evs[] = {&R.e_begin, &R.e_hist, &R.e_sorted, &R.e_end, &R.e_h2d0, &R.e_h2d1, &R.e_d2h0, &R.e_d2h1};
@@ -272,7 +272,7 @@ int radix_begin(msort_ctx* ctx, Rank& R, const void* src, uint64_t c) {
     CUDA_TRY(radix_prologue(src, c, ctx->kt, ws, R.st));
     ctx->tm.kernel_launches += 2;
     if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_hist, R.st));
-    if (ctx->skip_trivial) CUDA_TRY(cudaMemcpyAsync(R.h_trivial, ws.trivial, 16 * sizeof(uint32_t), cudaMemcpyDeviceToHost, R.st));
+    if (ctx->skip_trivial) CUDA_TRY(cudaMemcpyAsync(R.h_trivial, ws.trivial, 24 * sizeof(uint32_t), cudaMemcpyDeviceToHost, R.st));
     return MSORT_OK;
 }
 
@@ -311,12 +311,15 @@ int radix_passes(msort_ctx* ctx, Rank& R, const void* src, void* dst, void* tmp,
         // Ranking (flag 4 = one smem atomic per key): stable when the GPU passed
         // the lane-order self-test, and always valid for the first executed pass
         // (nothing has ordered the keys yet).  A skewed digit (one value holding
-        // more than 1/16 of the keys) makes same-address atomics serialize, so
-        // such passes rank by peer match instead (host knows the histogram when
-        // skip_trivial synchronised on it).
-        const bool skewed = ctx->skip_trivial && uint64_t(R.h_trivial[8 + R.pass_ids[j]]) * 16 > c;
-        const bool atomic_rank = !skewed && (j == 0 || atomic_rank_ok());
-        const int flags = (j == 0 ? 1 : 0) | (j == E - 1 ? 2 : 0) | (atomic_rank ? 4 : 0);
+        // more than 1/16 of the keys) would make same-address atomics serialize:
+        // its digit value goes to the kernel (flags bits 8.., value + 1), whose
+        // lanes on that digit reserve their slots with one atomic per warp row
+        // (host knows the histogram when skip_trivial synchronised on it).
+        const int pid = R.pass_ids[j];
+        const bool skewed = ctx->skip_trivial && uint64_t(R.h_trivial[8 + pid]) * 16 > c;
+        const bool atomic_rank = j == 0 || atomic_rank_ok();
+        const int hot = (skewed && atomic_rank) ? int(R.h_trivial[16 + pid] & 0xFF) + 1 : 0;
+        const int flags = (j == 0 ? 1 : 0) | (j == E - 1 ? 2 : 0) | (atomic_rank ? 4 : 0) | (hot << 8);
         if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_pass[j][0], R.st));
         CUDA_TRY(launch_onesweep(in, out, c, ctx->kt, R.pass_ids[j], flags, ws, ws.base + R.pass_ids[j] * 256, R.st));
         ctx->tm.kernel_launches += 1;

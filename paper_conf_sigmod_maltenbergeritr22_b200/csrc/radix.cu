@@ -107,7 +107,7 @@ __global__ void __launch_bounds__(kRadix) scan_kernel(const uint32_t* __restrict
                                                       uint32_t* __restrict__ trivial, uint64_t n) {
     __shared__ uint32_t wsum[kRadix / 32];
     __shared__ int any_full;
-    __shared__ uint32_t max_bin;
+    __shared__ unsigned long long max_bin;  // count << 8 | digit
     const int p = blockIdx.x, d = threadIdx.x, lane = d & 31, warp = d >> 5;
     if (d == 0) {
         any_full = 0;
@@ -126,11 +126,12 @@ __global__ void __launch_bounds__(kRadix) scan_kernel(const uint32_t* __restrict
     for (int w = 0; w < warp; ++w) pre += wsum[w];
     base[p * kRadix + d] = pre + x - v;
     if (uint64_t(v) == n) any_full = 1;
-    atomicMax(&max_bin, v);
+    atomicMax(&max_bin, (static_cast<unsigned long long>(v) << 8) | unsigned(d));
     __syncthreads();
     if (d == 0 && trivial) {
         trivial[p] = any_full;
-        trivial[8 + p] = max_bin;  // most frequent digit value of the pass (skew)
+        trivial[8 + p] = uint32_t(max_bin >> 8);     // size of the largest digit bin of the pass (skew)
+        trivial[16 + p] = uint32_t(max_bin & 0xFF);  // its digit value
     }
 }
 
@@ -212,7 +213,8 @@ template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg, bool STA
 __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     onesweep_kernel(const U* __restrict__ in, U* __restrict__ out, uint32_t n, uint32_t shift,
                     const uint32_t* __restrict__ base, unsigned long long* __restrict__ status,
-                    uint32_t* __restrict__ tile_counter, uint32_t tag, unsigned long long* __restrict__ gagg) {
+                    uint32_t* __restrict__ tile_counter, uint32_t tag, unsigned long long* __restrict__ gagg,
+                    uint32_t hot) {
     constexpr int THREADS = Cfg::kThreads;
     constexpr int ITEMS = Cfg::kItems;
     constexpr int WARPS = Cfg::kWarps;
@@ -473,6 +475,20 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
                 continue;
             }
             if constexpr (!STABLE) {
+                if (hot < kRadix) {
+                    // skewed pass (one digit holds > 1/16 of the keys): the lanes on
+                    // the hot digit reserve their slots with ONE atomic by the first
+                    // of them and rank by lane order (same-address atomics would be
+                    // served one lane at a time); the others take one atomic each
+                    const uint32_t hm = __ballot_sync(0xffffffffu, d == hot);
+                    const int first = hm ? __ffs(hm) - 1 : 0;
+                    uint32_t hb = 0;
+                    if (hm && lane == first) hb = atomicAdd(&s_cnt[warp][hot], uint32_t(__popc(hm)));
+                    hb = __shfl_sync(0xffffffffu, hb, first);
+                    const uint32_t slot = d == hot ? hb + __popc(hm & lt) : atomicAdd(&s_cnt[warp][d], 1u);
+                    s_keys[slot] = keys[i];
+                    continue;
+                }
                 s_keys[atomicAdd(&s_cnt[warp][d], 1u)] = keys[i];
                 continue;
             }
@@ -635,7 +651,7 @@ __global__ void __launch_bounds__(256) rank_probe_kernel(uint32_t seed, uint32_t
 
 template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg, bool STABLE>
 cudaError_t launch_onesweep_c(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
-                              const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
+                              const uint32_t* base_row, uint32_t tag, cudaStream_t st, uint32_t hot) {
     const size_t smem = Cfg::template smem_bytes<U>();
     auto kern = onesweep_kernel<U, FLOAT, ENC_IN, DEC_OUT, Cfg, STABLE>;
     // per-device attribute: set on every launch (cheap, and correct when one
@@ -651,35 +667,36 @@ cudaError_t launch_onesweep_c(const void* in, void* out, uint64_t n, int pass, c
     if (grid > tiles) grid = tiles;
     kern<<<unsigned(grid), Cfg::kThreads, smem, st>>>(reinterpret_cast<const U*>(in), reinterpret_cast<U*>(out),
                                                      uint32_t(n), uint32_t(8 * pass), base_row, ws.status,
-                                                     ws.counters + pass, tag, ws.gagg + size_t(pass) * ws.groups * kRadix);
+                                                     ws.counters + pass, tag, ws.gagg + size_t(pass) * ws.groups * kRadix,
+                                                     hot);
     return cudaGetLastError();
 }
 
 template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, bool STABLE>
 cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
-                              const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
+                              const uint32_t* base_row, uint32_t tag, cudaStream_t st, uint32_t hot) {
     const int c = env_cfg();
     if constexpr (sizeof(U) == 4) {
         switch (c) {
-            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_1, STABLE>(in, out, n, pass, ws, base_row, tag, st);
-            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_2, STABLE>(in, out, n, pass, ws, base_row, tag, st);
-            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_3, STABLE>(in, out, n, pass, ws, base_row, tag, st);
-            case 4: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_4, STABLE>(in, out, n, pass, ws, base_row, tag, st);
-            case 5: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_5, STABLE>(in, out, n, pass, ws, base_row, tag, st);
-            case 6: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_6, STABLE>(in, out, n, pass, ws, base_row, tag, st);
-            case 7: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_7, STABLE>(in, out, n, pass, ws, base_row, tag, st);
-            case 8: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_8, STABLE>(in, out, n, pass, ws, base_row, tag, st);
-            case 9: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_9, STABLE>(in, out, n, pass, ws, base_row, tag, st);
-            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_0, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_1, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_2, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_3, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            case 4: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_4, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            case 5: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_5, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            case 6: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_6, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            case 7: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_7, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            case 8: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_8, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            case 9: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_9, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
         }
     } else {
         switch (c) {
-            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_1, STABLE>(in, out, n, pass, ws, base_row, tag, st);
-            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_2, STABLE>(in, out, n, pass, ws, base_row, tag, st);
-            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_3, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_1, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_2, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_3, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
             case 4: case 5: case 6: case 7: case 8: case 9:
-                return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st);
-            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st);
+                return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
         }
     }
 }
@@ -687,23 +704,25 @@ cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, c
 template <typename U>
 cudaError_t launch_onesweep_int(const void* in, void* out, uint64_t n, int pass, int flags, const RadixWs& ws,
                                 const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
-    if (flags & 4) return launch_onesweep_t<U, false, false, false, false>(in, out, n, pass, ws, base_row, tag, st);
-    return launch_onesweep_t<U, false, false, false, true>(in, out, n, pass, ws, base_row, tag, st);
+    const uint32_t hot = (flags >> 8) & 0x1FF ? ((flags >> 8) & 0x1FF) - 1 : 0xFFFFFFFFu;
+    if (flags & 4) return launch_onesweep_t<U, false, false, false, false>(in, out, n, pass, ws, base_row, tag, st, hot);
+    return launch_onesweep_t<U, false, false, false, true>(in, out, n, pass, ws, base_row, tag, st, hot);
 }
 
 template <typename U>
 cudaError_t launch_onesweep_float(const void* in, void* out, uint64_t n, int pass, int flags, const RadixWs& ws,
                                   const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
+    const uint32_t hot = (flags >> 8) & 0x1FF ? ((flags >> 8) & 0x1FF) - 1 : 0xFFFFFFFFu;
     const bool enc = flags & 1, dec = flags & 2;
     const bool atom = flags & 4;
-    if (enc && dec && atom) return launch_onesweep_t<U, true, true, true, false>(in, out, n, pass, ws, base_row, tag, st);
-    if (dec && !enc && atom) return launch_onesweep_t<U, true, false, true, false>(in, out, n, pass, ws, base_row, tag, st);
-    if (!enc && !dec && atom) return launch_onesweep_t<U, true, false, false, false>(in, out, n, pass, ws, base_row, tag, st);
-    if (enc && dec) return launch_onesweep_t<U, true, true, true, true>(in, out, n, pass, ws, base_row, tag, st);
-    if (enc && (flags & 4)) return launch_onesweep_t<U, true, true, false, false>(in, out, n, pass, ws, base_row, tag, st);
-    if (enc) return launch_onesweep_t<U, true, true, false, true>(in, out, n, pass, ws, base_row, tag, st);
-    if (dec) return launch_onesweep_t<U, true, false, true, true>(in, out, n, pass, ws, base_row, tag, st);
-    return launch_onesweep_t<U, true, false, false, true>(in, out, n, pass, ws, base_row, tag, st);
+    if (enc && dec && atom) return launch_onesweep_t<U, true, true, true, false>(in, out, n, pass, ws, base_row, tag, st, hot);
+    if (dec && !enc && atom) return launch_onesweep_t<U, true, false, true, false>(in, out, n, pass, ws, base_row, tag, st, hot);
+    if (!enc && !dec && atom) return launch_onesweep_t<U, true, false, false, false>(in, out, n, pass, ws, base_row, tag, st, hot);
+    if (enc && dec) return launch_onesweep_t<U, true, true, true, true>(in, out, n, pass, ws, base_row, tag, st, hot);
+    if (enc && (flags & 4)) return launch_onesweep_t<U, true, true, false, false>(in, out, n, pass, ws, base_row, tag, st, hot);
+    if (enc) return launch_onesweep_t<U, true, true, false, true>(in, out, n, pass, ws, base_row, tag, st, hot);
+    if (dec) return launch_onesweep_t<U, true, false, true, true>(in, out, n, pass, ws, base_row, tag, st, hot);
+    return launch_onesweep_t<U, true, false, false, true>(in, out, n, pass, ws, base_row, tag, st, hot);
 }
 
 }  // namespace
@@ -725,7 +744,7 @@ uint32_t radix_tile_keys(int kt) { return key_bytes(kt) == 4 ? kMinTile32 : kMin
 
 static size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
-static size_t head_bytes() { return align_up(8 * 4 + 8 * 256 * 4 * 2 + 16 * 4, 256); }
+static size_t head_bytes() { return align_up(8 * 4 + 8 * 256 * 4 * 2 + 24 * 4, 256); }
 
 constexpr uint64_t kMinGroup = 8;  // smallest look-back group of the configs above (sizes the allocation)
 

@@ -7,7 +7,8 @@ import paper_conf_sigmod_maltenbergeritr22_b200 as ms
 from oracle import sort as osort
 def dev(a): return torch.from_numpy(a.view(np.uint8).copy()).cuda()
 ok = True
-for kt, n, g, ex in [("u32", 20011, 1, 0), ("f32", 30000, 4, 0), ("u64", 9001 * 2, 2, 1), ("u32", 24000, 4, 2)]:
+for kt, n, g, ex in [("u32", 20011, 1, 0), ("f32", 30000, 4, 0), ("u64", 9001 * 2, 2, 1), ("u32", 24000, 4, 2),
+                     ("u64", 16000, 8, 2), ("u32", 24000, 4, 3)]:
     a = mi.np_generate(n, kt, "uniform", seed=2)
     c = n // g
     ctx = ms.Context(g, n, kt, device_ids=[0] * g)
@@ -20,4 +21,21 @@ for kt, n, g, ex in [("u32", 20011, 1, 0), ("f32", 30000, 4, 0), ("u64", 9001 * 
     ok &= good
     print(kt, n, g, ex, "ok" if good else "MISMATCH", flush=True)
     ctx.close()
+# merge step on runs/output at odd key offsets (bulk copies over-fetch to 16-byte bounds)
+for kt, oa, ob, oo, al, bl in [("u32", 1, 3, 2, 9001, 7777), ("u64", 1, 0, 1, 5003, 6007)]:
+    K = mi.KEY_BYTES[kt]
+    a = osort.oracle_sort(mi.np_generate(al, kt, "uniform", seed=3), kt)
+    b = osort.oracle_sort(mi.np_generate(bl, kt, "uniform", seed=4), kt)
+    da = dev(np.concatenate([np.zeros(oa, a.dtype), a]))
+    db = dev(np.concatenate([np.zeros(ob, b.dtype), b]))
+    out = torch.zeros((al + bl + oo) * K, dtype=torch.uint8, device="cuda")
+    wsb = ms.msort_merge_workspace_bytes(al + bl, kt)
+    ws = torch.empty(wsb, dtype=torch.uint8, device="cuda")
+    ms.msort_step_merge(ms.tensor_ptr(da) + oa * K, al, ms.tensor_ptr(db) + ob * K, bl, ms.tensor_ptr(out) + oo * K, kt,
+                        ms.tensor_ptr(ws), wsb)
+    torch.cuda.synchronize()
+    got = out.cpu().numpy().view(mi.NP_DTYPE[kt])[oo:oo + al + bl]
+    good = np.array_equal(got.view(np.uint8), osort.oracle_sort(np.concatenate([a, b]), kt).view(np.uint8))
+    ok &= good
+    print("merge", kt, al, bl, "ok" if good else "MISMATCH", flush=True)
 print("ALL OK" if ok else "FAIL")
