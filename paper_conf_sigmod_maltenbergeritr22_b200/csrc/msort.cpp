@@ -276,6 +276,19 @@ int radix_begin(msort_ctx* ctx, Rank& R, const void* src, uint64_t c) {
     return MSORT_OK;
 }
 
+// skewed-pass ranking policy (MSORT_SKEW_MODE, tuning only): 0 = peer match for
+// every skewed pass, 1 = hot-digit atomics for every skewed pass, 2 (default) =
+// hot-digit atomics only when one digit holds > 1/4 of the keys
+int skew_mode() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = std::getenv("MSORT_SKEW_MODE");
+        v = e ? std::atoi(e) : 2;
+        if (v < 0 || v > 2) v = 2;
+    }
+    return v;
+}
+
 // src -> dst through tmp; an even number of executed passes, so the last write
 // lands in dst and no pass reads and writes the same buffer.
 int radix_passes(msort_ctx* ctx, Rank& R, const void* src, void* dst, void* tmp, uint64_t c) {
@@ -315,10 +328,18 @@ int radix_passes(msort_ctx* ctx, Rank& R, const void* src, void* dst, void* tmp,
         // its digit value goes to the kernel (flags bits 8.., value + 1), whose
         // lanes on that digit reserve their slots with one atomic per warp row
         // (host knows the histogram when skip_trivial synchronised on it).
+        // Measured (profiles/radix_tuning_r1.md): with a moderately hot digit
+        // (zipf, largest bin ~10%) several digits collide per warp row and the
+        // peer match wins; with a dominant digit (largest bin > 1/4) the hot-digit
+        // atomic ranking wins.
         const int pid = R.pass_ids[j];
-        const bool skewed = ctx->skip_trivial && uint64_t(R.h_trivial[8 + pid]) * 16 > c;
-        const bool atomic_rank = j == 0 || atomic_rank_ok();
-        const int hot = (skewed && atomic_rank) ? int(R.h_trivial[16 + pid] & 0xFF) + 1 : 0;
+        const uint64_t maxbin = ctx->skip_trivial ? uint64_t(R.h_trivial[8 + pid]) : 0;
+        const int mode = skew_mode();
+        const bool skewed = maxbin * 16 > c;
+        const bool dominant = mode == 1 ? skewed : (mode == 0 ? false : maxbin * 4 > c);
+        bool atomic_rank = j == 0 || atomic_rank_ok();
+        if (skewed && !dominant) atomic_rank = false;  // peer match
+        const int hot = (dominant && atomic_rank) ? int(R.h_trivial[16 + pid] & 0xFF) + 1 : 0;
         const int flags = (j == 0 ? 1 : 0) | (j == E - 1 ? 2 : 0) | (atomic_rank ? 4 : 0) | (hot << 8);
         if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_pass[j][0], R.st));
         CUDA_TRY(launch_onesweep(in, out, c, ctx->kt, R.pass_ids[j], flags, ws, ws.base + R.pass_ids[j] * 256, R.st));

@@ -6,7 +6,8 @@ Together these imply byte equality with the (unique) oracle result.
 
 configs[2]: 4e9 uniform u32 on one GPU (the bench's N=1 workload);
 configs[1]: 2^28 uniform u32 on 2 chunks (virtual ranks on one GPU);
-configs[3]/[4]: 2e9 keys on 8 chunks (virtual ranks), zipf u32 and f32.
+configs[3]/[4]: 2e9 keys on 8 chunks (virtual ranks): zipf / reverse / nearly-sorted u32, f32, u64, and
+NEXT-1 on zipf.
 """
 import os
 
@@ -107,18 +108,23 @@ def test_config3_4e9_u32_one_gpu():
     _check(chunks, n, "u32", "uniform", 1)
 
 
-@pytest.mark.parametrize("n,g,kt,dist", [
-    (1 << 28, 2, "u32", "uniform"),          # configs[1]
-    (2_000_000_000, 8, "u32", "zipf"),        # configs[3] (pivot imbalance stress)
-    (2_000_000_000, 8, "f32", "uniform"),     # configs[4] float keys
+@pytest.mark.parametrize("n,g,kt,dist,exchange", [
+    (1 << 28, 2, "u32", "uniform", 0),          # configs[1]
+    (2_000_000_000, 8, "u32", "zipf", 0),        # configs[3] (pivot imbalance stress)
+    (2_000_000_000, 8, "u32", "reverse", 0),     # configs[3]: x_d = c on every pair, every stage
+    (2_000_000_000, 8, "u32", "nearly", 0),      # configs[3]
+    (2_000_000_000, 8, "f32", "uniform", 0),     # configs[4] float keys
+    (2_000_000_000, 8, "u64", "uniform", 0),     # configs[4] 64-bit keys
+    (2_000_000_000, 8, "u32", "zipf", 2),        # NEXT-1 (fused all-to-all) at full size
 ])
-def test_p2p_virtual_full_size(n, g, kt, dist):
+def test_p2p_virtual_full_size(n, g, kt, dist, exchange):
     import paper_conf_sigmod_maltenbergeritr22_b200 as ms
     chunks, c = _gen_chunks(n, g, kt, dist, 3)
     ctx = ms.Context(g, n, kt, device_ids=[0] * g)
+    ctx.set_option(ms.MSORT_OPT_EXCHANGE, exchange)
     ctx.sort_device([ms.tensor_ptr(t) for t in chunks], c)
     torch.cuda.synchronize()
     tm = ctx.timings()
     ctx.close()
-    assert tm["n_stages"] == g - 1
+    assert tm["n_stages"] == (g - 1 if exchange < 2 else 1)
     _check(chunks, n, kt, dist, 3)
