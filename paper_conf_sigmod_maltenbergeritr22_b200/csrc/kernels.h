@@ -43,9 +43,10 @@ cudaError_t launch_scan(const uint32_t* hist, uint32_t* base, uint32_t* trivial,
 bool atomic_rank_ok();
 // one onesweep pass; flags: 1 = encode on load, 2 = decode on store,
 // 4 = atomic ranking (always valid for the first pass; used for every pass when
-// atomic_rank_ok())
+// atomic_rank_ok()), 8 = skewed pass: with atomic ranking, the 4 digit values in
+// `hot` (one per byte) are ranked with one atomic per warp row and digit
 cudaError_t launch_onesweep(const void* in, void* out, uint64_t n, int kt, int pass, int flags, const RadixWs& ws,
-                            const uint32_t* base_row, cudaStream_t st);
+                            const uint32_t* base_row, cudaStream_t st, uint32_t hot = 0);
 
 // ----- merge phase (S4-S6) -------------------------------------------------
 struct GroupPtrs {

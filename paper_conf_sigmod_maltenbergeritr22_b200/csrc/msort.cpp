@@ -276,9 +276,9 @@ int radix_begin(msort_ctx* ctx, Rank& R, const void* src, uint64_t c) {
     return MSORT_OK;
 }
 
-// skewed-pass ranking policy (MSORT_SKEW_MODE, tuning only): 0 = peer match for
-// every skewed pass, 1 = hot-digit atomics for every skewed pass, 2 (default) =
-// hot-digit atomics only when one digit holds > 1/4 of the keys
+// skewed-pass ranking (MSORT_SKEW_MODE, tuning only): 0 = peer match, 1 = one
+// atomic per warp row for each of the 4 most frequent digit values, 2 (default)
+// = 1 when one digit holds > 1/4 of the keys, else 0
 int skew_mode() {
     static int v = -1;
     if (v < 0) {
@@ -328,21 +328,22 @@ int radix_passes(msort_ctx* ctx, Rank& R, const void* src, void* dst, void* tmp,
         // its digit value goes to the kernel (flags bits 8.., value + 1), whose
         // lanes on that digit reserve their slots with one atomic per warp row
         // (host knows the histogram when skip_trivial synchronised on it).
-        // Measured (profiles/radix_tuning_r1.md): with a moderately hot digit
-        // (zipf, largest bin ~10%) several digits collide per warp row and the
-        // peer match wins; with a dominant digit (largest bin > 1/4) the hot-digit
-        // atomic ranking wins.
+        // Skewed passes (profiles/radix_tuning_r1.md): a dominant digit (largest
+        // bin > 1/4 of the keys) -> the 4 most frequent digit values are ranked
+        // with one atomic per warp row each (flag 8); moderate skew (zipf: ~100
+        // elevated digits, the largest ~12%) -> peer match, which handles every
+        // colliding digit.  MSORT_SKEW_MODE 0 / 1 forces peer match / flag 8.
         const int pid = R.pass_ids[j];
         const uint64_t maxbin = ctx->skip_trivial ? uint64_t(R.h_trivial[8 + pid]) : 0;
-        const int mode = skew_mode();
         const bool skewed = maxbin * 16 > c;
+        const int mode = skew_mode();
         const bool dominant = mode == 1 ? skewed : (mode == 0 ? false : maxbin * 4 > c);
         bool atomic_rank = j == 0 || atomic_rank_ok();
         if (skewed && !dominant) atomic_rank = false;  // peer match
-        const int hot = (dominant && atomic_rank) ? int(R.h_trivial[16 + pid] & 0xFF) + 1 : 0;
-        const int flags = (j == 0 ? 1 : 0) | (j == E - 1 ? 2 : 0) | (atomic_rank ? 4 : 0) | (hot << 8);
+        const bool hot = dominant && atomic_rank;
+        const int flags = (j == 0 ? 1 : 0) | (j == E - 1 ? 2 : 0) | (atomic_rank ? 4 : 0) | (hot ? 8 : 0);
         if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_pass[j][0], R.st));
-        CUDA_TRY(launch_onesweep(in, out, c, ctx->kt, R.pass_ids[j], flags, ws, ws.base + R.pass_ids[j] * 256, R.st));
+        CUDA_TRY(launch_onesweep(in, out, c, ctx->kt, pid, flags, ws, ws.base + pid * 256, R.st, R.h_trivial[16 + pid]));
         ctx->tm.kernel_launches += 1;
         if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_pass[j][1], R.st));
         in = out;

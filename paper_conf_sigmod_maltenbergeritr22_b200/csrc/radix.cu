@@ -126,12 +126,25 @@ __global__ void __launch_bounds__(kRadix) scan_kernel(const uint32_t* __restrict
     for (int w = 0; w < warp; ++w) pre += wsum[w];
     base[p * kRadix + d] = pre + x - v;
     if (uint64_t(v) == n) any_full = 1;
-    atomicMax(&max_bin, (static_cast<unsigned long long>(v) << 8) | unsigned(d));
-    __syncthreads();
+    // the 4 most frequent digit values (skewed passes rank them with one atomic
+    // per warp row each), largest first
+    uint32_t top4 = 0, top_count = 0;
+    bool taken = false;
+    for (int q = 0; q < 4; ++q) {
+        if (!taken) atomicMax(&max_bin, (static_cast<unsigned long long>(v) << 8) | unsigned(d));
+        __syncthreads();
+        const unsigned long long b = max_bin;
+        if (q == 0) top_count = uint32_t(b >> 8);
+        top4 |= uint32_t(b & 0xFF) << (8 * q);
+        if (uint32_t(b & 0xFF) == uint32_t(d)) taken = true;
+        __syncthreads();
+        if (d == 0) max_bin = 0;
+        __syncthreads();
+    }
     if (d == 0 && trivial) {
         trivial[p] = any_full;
-        trivial[8 + p] = uint32_t(max_bin >> 8);     // size of the largest digit bin of the pass (skew)
-        trivial[16 + p] = uint32_t(max_bin & 0xFF);  // its digit value
+        trivial[8 + p] = top_count;  // size of the largest digit bin of the pass (skew)
+        trivial[16 + p] = top4;      // the 4 most frequent digit values, one per byte
     }
 }
 
@@ -214,7 +227,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     onesweep_kernel(const U* __restrict__ in, U* __restrict__ out, uint32_t n, uint32_t shift,
                     const uint32_t* __restrict__ base, unsigned long long* __restrict__ status,
                     uint32_t* __restrict__ tile_counter, uint32_t tag, unsigned long long* __restrict__ gagg,
-                    uint32_t hot) {
+                    uint32_t hot, bool hot_on) {
     constexpr int THREADS = Cfg::kThreads;
     constexpr int ITEMS = Cfg::kItems;
     constexpr int WARPS = Cfg::kWarps;
@@ -475,18 +488,24 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
                 continue;
             }
             if constexpr (!STABLE) {
-                if (hot < kRadix) {
-                    // skewed pass (one digit holds > 1/16 of the keys): the lanes on
-                    // the hot digit reserve their slots with ONE atomic by the first
-                    // of them and rank by lane order (same-address atomics would be
-                    // served one lane at a time); the others take one atomic each
-                    const uint32_t hm = __ballot_sync(0xffffffffu, d == hot);
-                    const int first = hm ? __ffs(hm) - 1 : 0;
-                    uint32_t hb = 0;
-                    if (hm && lane == first) hb = atomicAdd(&s_cnt[warp][hot], uint32_t(__popc(hm)));
-                    hb = __shfl_sync(0xffffffffu, hb, first);
-                    const uint32_t slot = d == hot ? hb + __popc(hm & lt) : atomicAdd(&s_cnt[warp][d], 1u);
-                    s_keys[slot] = keys[i];
+                if (hot_on) {
+                    // skewed pass: the lanes on one of the 4 most frequent digits
+                    // (`hot`, one per byte) reserve their slots with one atomic by
+                    // the first lane of their group and rank by lane order (ballot);
+                    // every other lane takes one atomic itself - all in ONE atomic
+                    // instruction, so no digit value piles up on one address
+                    uint32_t mine = 0;
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        const uint32_t h = (hot >> (8 * q)) & 0xFFu;
+                        const uint32_t m = __ballot_sync(0xffffffffu, d == h);
+                        if (d == h) mine = m;
+                    }
+                    const int first = mine ? __ffs(mine) - 1 : lane;
+                    uint32_t got = 0;
+                    if (!mine || lane == first) got = atomicAdd(&s_cnt[warp][d], mine ? uint32_t(__popc(mine)) : 1u);
+                    got = __shfl_sync(0xffffffffu, got, first);
+                    s_keys[got + __popc(mine & lt)] = keys[i];
                     continue;
                 }
                 s_keys[atomicAdd(&s_cnt[warp][d], 1u)] = keys[i];
@@ -651,7 +670,7 @@ __global__ void __launch_bounds__(256) rank_probe_kernel(uint32_t seed, uint32_t
 
 template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg, bool STABLE>
 cudaError_t launch_onesweep_c(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
-                              const uint32_t* base_row, uint32_t tag, cudaStream_t st, uint32_t hot) {
+                              const uint32_t* base_row, uint32_t tag, cudaStream_t st, uint32_t hot, bool hot_on) {
     const size_t smem = Cfg::template smem_bytes<U>();
     auto kern = onesweep_kernel<U, FLOAT, ENC_IN, DEC_OUT, Cfg, STABLE>;
     // per-device attribute: set on every launch (cheap, and correct when one
@@ -668,61 +687,61 @@ cudaError_t launch_onesweep_c(const void* in, void* out, uint64_t n, int pass, c
     kern<<<unsigned(grid), Cfg::kThreads, smem, st>>>(reinterpret_cast<const U*>(in), reinterpret_cast<U*>(out),
                                                      uint32_t(n), uint32_t(8 * pass), base_row, ws.status,
                                                      ws.counters + pass, tag, ws.gagg + size_t(pass) * ws.groups * kRadix,
-                                                     hot);
+                                                     hot, hot_on);
     return cudaGetLastError();
 }
 
 template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, bool STABLE>
 cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
-                              const uint32_t* base_row, uint32_t tag, cudaStream_t st, uint32_t hot) {
+                              const uint32_t* base_row, uint32_t tag, cudaStream_t st, uint32_t hot, bool hot_on) {
     const int c = env_cfg();
     if constexpr (sizeof(U) == 4) {
         switch (c) {
-            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_1, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
-            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_2, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
-            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_3, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
-            case 4: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_4, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
-            case 5: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_5, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
-            case 6: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_6, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
-            case 7: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_7, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
-            case 8: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_8, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
-            case 9: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_9, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
-            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_1, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_2, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_3, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 4: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_4, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 5: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_5, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 6: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_6, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 7: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_7, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 8: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_8, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 9: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_9, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
         }
     } else {
         switch (c) {
-            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_1, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
-            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_2, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
-            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_3, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_1, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_2, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_3, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
             case 4: case 5: case 6: case 7: case 8: case 9:
-                return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
-            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot);
+                return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
         }
     }
 }
 
 template <typename U>
 cudaError_t launch_onesweep_int(const void* in, void* out, uint64_t n, int pass, int flags, const RadixWs& ws,
-                                const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
-    const uint32_t hot = (flags >> 8) & 0x1FF ? ((flags >> 8) & 0x1FF) - 1 : 0xFFFFFFFFu;
-    if (flags & 4) return launch_onesweep_t<U, false, false, false, false>(in, out, n, pass, ws, base_row, tag, st, hot);
-    return launch_onesweep_t<U, false, false, false, true>(in, out, n, pass, ws, base_row, tag, st, hot);
+                                const uint32_t* base_row, uint32_t tag, cudaStream_t st, uint32_t hot) {
+    const bool hot_on = flags & 8;
+    if (flags & 4) return launch_onesweep_t<U, false, false, false, false>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+    return launch_onesweep_t<U, false, false, false, true>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
 }
 
 template <typename U>
 cudaError_t launch_onesweep_float(const void* in, void* out, uint64_t n, int pass, int flags, const RadixWs& ws,
-                                  const uint32_t* base_row, uint32_t tag, cudaStream_t st) {
-    const uint32_t hot = (flags >> 8) & 0x1FF ? ((flags >> 8) & 0x1FF) - 1 : 0xFFFFFFFFu;
+                                  const uint32_t* base_row, uint32_t tag, cudaStream_t st, uint32_t hot) {
+    const bool hot_on = flags & 8;
     const bool enc = flags & 1, dec = flags & 2;
     const bool atom = flags & 4;
-    if (enc && dec && atom) return launch_onesweep_t<U, true, true, true, false>(in, out, n, pass, ws, base_row, tag, st, hot);
-    if (dec && !enc && atom) return launch_onesweep_t<U, true, false, true, false>(in, out, n, pass, ws, base_row, tag, st, hot);
-    if (!enc && !dec && atom) return launch_onesweep_t<U, true, false, false, false>(in, out, n, pass, ws, base_row, tag, st, hot);
-    if (enc && dec) return launch_onesweep_t<U, true, true, true, true>(in, out, n, pass, ws, base_row, tag, st, hot);
-    if (enc && (flags & 4)) return launch_onesweep_t<U, true, true, false, false>(in, out, n, pass, ws, base_row, tag, st, hot);
-    if (enc) return launch_onesweep_t<U, true, true, false, true>(in, out, n, pass, ws, base_row, tag, st, hot);
-    if (dec) return launch_onesweep_t<U, true, false, true, true>(in, out, n, pass, ws, base_row, tag, st, hot);
-    return launch_onesweep_t<U, true, false, false, true>(in, out, n, pass, ws, base_row, tag, st, hot);
+    if (enc && dec && atom) return launch_onesweep_t<U, true, true, true, false>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+    if (dec && !enc && atom) return launch_onesweep_t<U, true, false, true, false>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+    if (!enc && !dec && atom) return launch_onesweep_t<U, true, false, false, false>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+    if (enc && dec) return launch_onesweep_t<U, true, true, true, true>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+    if (enc && (flags & 4)) return launch_onesweep_t<U, true, true, false, false>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+    if (enc) return launch_onesweep_t<U, true, true, false, true>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+    if (dec) return launch_onesweep_t<U, true, false, true, true>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+    return launch_onesweep_t<U, true, false, false, true>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
 }
 
 }  // namespace
@@ -837,15 +856,15 @@ cudaError_t radix_prologue(const void* keys, uint64_t n, int kt, const RadixWs& 
 }
 
 cudaError_t launch_onesweep(const void* in, void* out, uint64_t n, int kt, int pass, int flags, const RadixWs& ws,
-                            const uint32_t* base_row, cudaStream_t st) {
+                            const uint32_t* base_row, cudaStream_t st, uint32_t hot) {
     if (n == 0) return cudaSuccess;
     // status words of other passes and of earlier sorts (epochs) are ignored
     const uint32_t tag = ((ws.epoch << 4) + uint32_t(pass) + 1) & 0x3FFFFFFFu;
     switch (kt) {
-        case 0: return launch_onesweep_int<uint32_t>(in, out, n, pass, flags, ws, base_row, tag, st);
-        case 1: return launch_onesweep_int<uint64_t>(in, out, n, pass, flags, ws, base_row, tag, st);
-        case 2: return launch_onesweep_float<uint32_t>(in, out, n, pass, flags, ws, base_row, tag, st);
-        case 3: return launch_onesweep_float<uint64_t>(in, out, n, pass, flags, ws, base_row, tag, st);
+        case 0: return launch_onesweep_int<uint32_t>(in, out, n, pass, flags, ws, base_row, tag, st, hot);
+        case 1: return launch_onesweep_int<uint64_t>(in, out, n, pass, flags, ws, base_row, tag, st, hot);
+        case 2: return launch_onesweep_float<uint32_t>(in, out, n, pass, flags, ws, base_row, tag, st, hot);
+        case 3: return launch_onesweep_float<uint64_t>(in, out, n, pass, flags, ws, base_row, tag, st, hot);
         default: return cudaErrorInvalidValue;
     }
 }
