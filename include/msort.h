@@ -116,7 +116,12 @@ enum {
                                        from the peers' chunks over NVLink;
                                        3: NEXT-1 with the exchange as separate pulls (every GPU copies its run
                                        from every chunk into a local buffer), then the merge tree            */
-    MSORT_OPT_SKIP_TRIVIAL = 2   /* 1: skip radix passes whose digit is constant (identity permutation)   */
+    MSORT_OPT_SKIP_TRIVIAL = 2,  /* 1: skip radix passes whose digit is constant (identity permutation)   */
+    MSORT_OPT_HOST_PIPELINE = 3  /* 1 (default): msort_sort_host on ONE GPU overlaps the transfers with the
+                                       sort - the chunk arrives in 4 pieces, each radix sorted while the next
+                                       is in flight, the sorted pieces merge, and the final merge runs in
+                                       slices, each copied back while the next one merges (chunks of at
+                                       least 2^20 keys); 0: H2D, sort, D2H one after the other           */
 };
 int msort_set_option(msort_ctx* ctx, int option, int64_t value);
 

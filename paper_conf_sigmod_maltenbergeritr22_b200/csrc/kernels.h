@@ -62,6 +62,10 @@ cudaError_t launch_splitters(const GroupPtrs& all, int g, uint64_t c, int kt, ui
 size_t merge_ws_bytes(uint64_t total, int kt);
 cudaError_t launch_merge(const void* a, uint64_t al, const void* b, uint64_t bl, void* out, int kt, void* ws,
                          cudaStream_t st, int* launches);
+// merge-path co-ranks: d_part[j] = a-elements among the first min(j*step, al+bl)
+// outputs of merging a and b (a wins ties), j < nparts
+cudaError_t launch_corank(const void* a, uint64_t al, const void* b, uint64_t bl, uint64_t step, uint64_t nparts,
+                          int kt, uint64_t* d_part, cudaStream_t st);
 // fill count keys with the largest key under T (tail padding, reading Q3)
 cudaError_t launch_fill_max(void* p, uint64_t count, int kt, cudaStream_t st);
 

@@ -797,6 +797,20 @@ cudaError_t launch_merge(const void* a, uint64_t al, const void* b, uint64_t bl,
     }
 }
 
+cudaError_t launch_corank(const void* a, uint64_t al, const void* b, uint64_t bl, uint64_t step, uint64_t nparts,
+                          int kt, uint64_t* d_part, cudaStream_t st) {
+    if (nparts == 0) return cudaSuccess;
+    const unsigned blocks = unsigned((nparts + 255) / 256);
+    switch (kt) {
+        case 0: partition_thread_kernel<uint32_t, false><<<blocks, 256, 0, st>>>((const uint32_t*)a, al, (const uint32_t*)b, bl, step, nparts, d_part); break;
+        case 1: partition_thread_kernel<uint64_t, false><<<blocks, 256, 0, st>>>((const uint64_t*)a, al, (const uint64_t*)b, bl, step, nparts, d_part); break;
+        case 2: partition_thread_kernel<uint32_t, true><<<blocks, 256, 0, st>>>((const uint32_t*)a, al, (const uint32_t*)b, bl, step, nparts, d_part); break;
+        case 3: partition_thread_kernel<uint64_t, true><<<blocks, 256, 0, st>>>((const uint64_t*)a, al, (const uint64_t*)b, bl, step, nparts, d_part); break;
+        default: return cudaErrorInvalidValue;
+    }
+    return cudaGetLastError();
+}
+
 cudaError_t launch_fill_max(void* p, uint64_t count, int kt, cudaStream_t st) {
     if (count == 0) return cudaSuccess;
     const unsigned blocks = unsigned(count < 256 * 1024 ? (count + 255) / 256 : 1024);

@@ -124,6 +124,9 @@ uint64_t chunk_size(uint64_t n, int g) {
 // ---------------------------------------------------------------------------
 // Per-rank state
 // ---------------------------------------------------------------------------
+constexpr int kPieces = 4;   // pipelined host sort: H2D pieces, each sorted while the next one arrives
+constexpr int kSlices = 4;   // ... and final-merge slices, each copied back while the next one merges
+
 struct Rank {
     int dev = 0;
     cudaStream_t st = nullptr;
@@ -141,6 +144,11 @@ struct Rank {
     cudaEvent_t e_begin = nullptr, e_hist = nullptr, e_sorted = nullptr, e_end = nullptr;
     cudaEvent_t e_h2d0 = nullptr, e_h2d1 = nullptr, e_d2h0 = nullptr, e_d2h1 = nullptr;
     cudaEvent_t e_pass[8][2] = {};
+    // pipelined host sort (g == 1): copy stream, piece arrivals, merged slices
+    cudaStream_t cst = nullptr;
+    cudaEvent_t e_piece[kPieces] = {};
+    cudaEvent_t e_slice[kSlices] = {};
+    cudaEvent_t e_merged = nullptr;
     cudaEvent_t e_sync[MSORT_MAX_STAGES + 1] = {};
     cudaEvent_t e_stage[MSORT_MAX_STAGES][2] = {};
     cudaEvent_t e_xch[MSORT_MAX_STAGES][2] = {};
@@ -184,6 +192,7 @@ struct msort_ctx {
     int timing = 1;
     int exchange = 0;
     int skip_trivial = 1;
+    int host_pipeline = 1;
     msort_timings tm{};
 };
 
@@ -194,6 +203,10 @@ int alloc_rank(msort_ctx* ctx, Rank& R, bool need_b1, bool need_stage) {
     CUDA_TRY(cudaSetDevice(R.dev));
     atomic_rank_ok();  // one-time per-device probe, outside any sort
     CUDA_TRY(cudaStreamCreateWithFlags(&R.st, cudaStreamNonBlocking));
+    CUDA_TRY(cudaStreamCreateWithFlags(&R.cst, cudaStreamNonBlocking));
+    for (auto& e : R.e_piece) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    for (auto& e : R.e_slice) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    CUDA_TRY(cudaEventCreate(&R.e_merged));
     const size_t bytes = std::max<size_t>(ctx->cap * K, 256);
     CUDA_TRY(cudaMalloc(&R.buf[0], bytes));
     if (need_b1) CUDA_TRY(cudaMalloc(&R.buf[1], bytes));
@@ -249,6 +262,15 @@ void free_rank(Rank& R) {
     for (auto& xe : R.e_xch)
         for (auto e : xe)
             if (e) cudaEventDestroy(e);
+    for (auto e : R.e_piece)
+        if (e) cudaEventDestroy(e);
+    for (auto e : R.e_slice)
+        if (e) cudaEventDestroy(e);
+    if (R.e_merged) cudaEventDestroy(R.e_merged);
+    if (R.cst) {
+        cudaStreamSynchronize(R.cst);
+        cudaStreamDestroy(R.cst);
+    }
     cudaStreamDestroy(R.st);
     R = Rank();
 }
@@ -926,6 +948,7 @@ int msort_set_option(msort_ctx* ctx, int option, int64_t value) {
     switch (option) {
         case MSORT_OPT_TIMING: ctx->timing = value ? 1 : 0; return MSORT_OK;
         case MSORT_OPT_SKIP_TRIVIAL: ctx->skip_trivial = value ? 1 : 0; return MSORT_OK;
+        case MSORT_OPT_HOST_PIPELINE: ctx->host_pipeline = value ? 1 : 0; return MSORT_OK;
         case MSORT_OPT_EXCHANGE:
             if (value < 0 || value > 3) return set_error(MSORT_ERR_INVALID_ARGUMENT, "exchange mode 0, 1, 2 or 3");
             if (value == 1)
@@ -1002,6 +1025,104 @@ int msort_sort_device(msort_ctx* ctx, void* const* chunks, uint64_t keys_per_gpu
     return MSORT_OK;
 }
 
+// End-to-end sort on one GPU with the transfers overlapped (S0/S8 around
+// S1-S3; the paper finds the transfers dominate).
+// The chunk arrives in kPieces pieces on the copy stream; each piece is radix
+// sorted (in place, B0 as scratch) as soon as it has landed, while the next
+// one is still in flight.  Pieces 0+1 merge into B0 while pieces 2-3 arrive,
+// pieces 2+3 merge after the last one; the final merge of the two runs is cut
+// into growing output ranges at merge-path co-ranks, and every slice is copied
+// back while the next one merges.  The pieces shrink (3/8, 3/8, 3/16, 1/16 of
+// the chunk) so that little sorting and merging is left once the last byte
+// has arrived.  Same result as the sequential path (a sort is unique).
+static constexpr uint64_t kPipeMinKeys = 1ull << 20;
+
+static int sort_host_pipelined(msort_ctx* ctx, char* host, uint64_t n, uint64_t c) {
+    Rank& R = ctx->r[0];
+    const size_t K = key_bytes(ctx->kt);
+    CUDA_TRY(cudaSetDevice(R.dev));
+    for (bool& b : R.xch_rec) b = false;
+    char* stage = static_cast<char*>(R.stage);
+    char* b0 = static_cast<char*>(R.buf[0]);
+    auto cut = [&](uint64_t num, uint64_t den) { return c * num / den / 1024 * 1024; };
+    const uint64_t pb[kPieces + 1] = {0, cut(3, 8), cut(6, 8), cut(15, 16), c};
+    // S0: every piece's H2D (and the tail padding, reading Q3) on the copy stream
+    CUDA_TRY(cudaEventRecord(R.e_h2d0, R.cst));
+    for (int i = 0; i < kPieces; ++i) {
+        const uint64_t lo = std::min(pb[i], n), hi = std::min(pb[i + 1], n);
+        if (hi > lo) CUDA_TRY(cudaMemcpyAsync(stage + lo * K, host + lo * K, (hi - lo) * K, cudaMemcpyHostToDevice, R.cst));
+        if (i == kPieces - 1 && c > n) {
+            CUDA_TRY(launch_fill_max(stage + n * K, c - n, ctx->kt, R.cst));
+            ctx->tm.kernel_launches += 1;
+        }
+        CUDA_TRY(cudaEventRecord(R.e_piece[i], R.cst));
+    }
+    CUDA_TRY(cudaEventRecord(R.e_h2d1, R.cst));
+    // S1-S3 per piece on the compute stream, round-1 merges as soon as possible
+    CUDA_TRY(cudaEventRecord(R.e_begin, R.st));
+    for (int i = 0; i < kPieces; ++i) {
+        const uint64_t len = pb[i + 1] - pb[i];
+        char* p = stage + pb[i] * K;
+        CUDA_TRY(cudaStreamWaitEvent(R.st, R.e_piece[i], 0));
+        MSORT_TRY(radix_begin(ctx, R, p, len));
+        if (ctx->skip_trivial) CUDA_TRY(cudaStreamSynchronize(R.st));
+        MSORT_TRY(radix_passes(ctx, R, p, p, b0 + pb[i] * K, len));
+        if (i == 1 || i == 3) {  // merge pieces i-1 and i into B0 (the radix scratch of later pieces lies past them)
+            const uint64_t a0 = pb[i - 1];
+            CUDA_TRY(launch_merge(stage + a0 * K, pb[i] - a0, p, len, b0 + a0 * K, ctx->kt, R.mws, R.st,
+                                  &ctx->tm.kernel_launches));
+        }
+        if (i == kPieces - 1) CUDA_TRY(cudaEventRecord(R.e_sorted, R.st));
+    }
+    CUDA_TRY(cudaEventRecord(R.e_merged, R.st));
+    // S8 overlapped with the final merge: slice co-ranks, then merge + D2H per slice
+    const char* A = b0;
+    const uint64_t al = pb[2];
+    const char* B = b0 + pb[2] * K;
+    const uint64_t bl = c - pb[2];
+    // co-ranks at multiples of c/64; slices end at 1/64, 1/16, 1/4 and all of
+    // the chunk: each copy (PCIe) outlasts the next slice's merge (HBM), so the
+    // copies run back to back and only the first, small merge is exposed
+    const uint64_t step = (c + 63) / 64 / 1024 * 1024 + 1024;
+    const int nsteps = int((c + step - 1) / step);
+    CUDA_TRY(launch_corank(A, al, B, bl, step, uint64_t(nsteps) + 1, ctx->kt, R.d_pivot, R.st));
+    ctx->tm.kernel_launches += 1;
+    CUDA_TRY(cudaMemcpyAsync(R.h_pivot, R.d_pivot, size_t(nsteps + 1) * sizeof(uint64_t), cudaMemcpyDeviceToHost, R.st));
+    CUDA_TRY(cudaStreamSynchronize(R.st));
+    int ends[kSlices], ns = 0;
+    for (int e : {1, 4, 16, nsteps})
+        if (e <= nsteps && (ns == 0 || e > ends[ns - 1])) ends[ns++] = e;
+    for (int s = 0; s < ns; ++s) {
+        const int j0 = s ? ends[s - 1] : 0, j1 = ends[s];
+        const uint64_t lo = uint64_t(j0) * step, hi = std::min(c, uint64_t(j1) * step);
+        const uint64_t a0 = R.h_pivot[j0], a1 = R.h_pivot[j1];
+        const uint64_t b0i = lo - a0, b1i = hi - a1;
+        CUDA_TRY(launch_merge(A + a0 * K, a1 - a0, B + b0i * K, b1i - b0i, stage + lo * K, ctx->kt, R.mws, R.st,
+                              &ctx->tm.kernel_launches));
+        CUDA_TRY(cudaEventRecord(R.e_slice[s], R.st));
+        CUDA_TRY(cudaStreamWaitEvent(R.cst, R.e_slice[s], 0));
+        if (s == 0) CUDA_TRY(cudaEventRecord(R.e_d2h0, R.cst));
+        const uint64_t dhi = std::min(hi, n);
+        if (dhi > lo) CUDA_TRY(cudaMemcpyAsync(host + lo * K, stage + lo * K, (dhi - lo) * K, cudaMemcpyDeviceToHost, R.cst));
+    }
+    CUDA_TRY(cudaEventRecord(R.e_end, R.st));
+    CUDA_TRY(cudaEventRecord(R.e_d2h1, R.cst));
+    CUDA_TRY(cudaEventSynchronize(R.e_d2h1));
+    CUDA_TRY(cudaEventSynchronize(R.e_end));
+    collect_timings(ctx, 1);
+    // phases overlap here: h2d = all pieces landed, sort = first piece's sort
+    // start .. last piece sorted, merge = .. final merge done, d2h = first
+    // slice's copy start .. last byte back
+    msort_timings& t = ctx->tm;
+    t.sort_ms = elapsed(R.e_begin, R.e_sorted);
+    t.merge_ms = elapsed(R.e_sorted, R.e_end);
+    t.h2d_ms = elapsed(R.e_h2d0, R.e_h2d1);
+    t.d2h_ms = elapsed(R.e_d2h0, R.e_d2h1);
+    t.total_ms = elapsed(R.e_h2d0, R.e_d2h1);
+    t.hist_ms = 0;  // (pass_ms_sum / passes_run: those of the last piece)
+    return MSORT_OK;
+}
+
 int msort_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n) {
     if (!ctx || ctx->dist) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL or dist ctx");
     if (n && !host_keys) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL keys");
@@ -1013,6 +1134,7 @@ int msort_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n) {
     reset_timings(ctx, c);
     const size_t K = key_bytes(ctx->kt);
     char* host = static_cast<char*>(host_keys);
+    if (g == 1 && ctx->host_pipeline && c >= kPipeMinKeys) return sort_host_pipelined(ctx, host, n, c);
     for (int i = 0; i < g; ++i) {
         Rank& R = ctx->r[i];
         CUDA_TRY(cudaSetDevice(R.dev));

@@ -108,6 +108,23 @@ def test_config3_4e9_u32_one_gpu():
     _check(chunks, n, "u32", "uniform", 1)
 
 
+def test_config3_4e9_u32_one_gpu_end_to_end():
+    """configs[2] end to end (bench.py's e2e call): pinned host keys -> msort_sort_host
+    (pipelined transfers, MSORT_OPT_HOST_PIPELINE default) -> host; checked on the GPU."""
+    import paper_conf_sigmod_maltenbergeritr22_b200 as ms
+    n = 4_000_000_000
+    chunks, c = _gen_chunks(n, 1, "u32", "uniform", 1)
+    host = torch.empty(n, dtype=chunks[0].dtype, pin_memory=True)
+    host.copy_(chunks[0][:n])
+    ctx = ms.Context(1, n, "u32", device_ids=[0])
+    ctx.sort_host(ms.tensor_ptr(host), n)
+    ctx.close()
+    chunks[0][:n].copy_(host)
+    del host
+    torch.cuda.synchronize()
+    _check(chunks, n, "u32", "uniform", 1)
+
+
 @pytest.mark.parametrize("n,g,kt,dist,exchange", [
     (1 << 28, 2, "u32", "uniform", 0),          # configs[1]
     (2_000_000_000, 8, "u32", "zipf", 0),        # configs[3] (pivot imbalance stress)

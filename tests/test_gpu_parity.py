@@ -288,6 +288,25 @@ def test_sort_host_end_to_end(ms, g, n):
     assert np.array_equal(h.numpy(), sort.oracle_sort(a, "u32"))
 
 
+@pytest.mark.parametrize("kt,dist,n", [("u32", "uniform", (1 << 22) + 3), ("u32", "zipf", (1 << 21) + 1),
+                                       ("u32", "reverse", 1 << 20), ("u64", "uniform", (1 << 21) + 2),
+                                       ("f32", "uniform", 3_000_001), ("f64", "uniform", (1 << 20) + 7)])
+@pytest.mark.parametrize("pipeline", [1, 0])
+def test_sort_host_pipelined(ms, kt, dist, n, pipeline):
+    """msort_sort_host on one GPU with MSORT_OPT_HOST_PIPELINE (4 pieces sorted as
+    they land, merged, the final merge sliced and copied back slice by slice) and
+    without it: both equal the oracle (the sorted multiset is unique, §8(c))."""
+    a = mi.np_generate(n, kt, dist, seed=5)
+    h = torch.from_numpy(a.copy()).pin_memory()
+    ctx = ms.Context(1, n, kt, device_ids=[0])
+    ctx.set_option(ms.MSORT_OPT_HOST_PIPELINE, pipeline)
+    ctx.sort_host(ms.tensor_ptr(h), n)
+    t = ctx.timings()
+    ctx.close()
+    assert bits(h.numpy(), kt).tobytes() == bits(sort.oracle_sort(a, kt), kt).tobytes()
+    assert t["total_ms"] > 0 and t["h2d_ms"] > 0 and t["d2h_ms"] > 0
+
+
 def test_msort_sort_host_pointer(ms):
     n = 100003
     a = mi.np_generate(n, "f32", "uniform", seed=9)
