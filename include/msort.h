@@ -117,11 +117,13 @@ enum {
                                        3: NEXT-1 with the exchange as separate pulls (every GPU copies its run
                                        from every chunk into a local buffer), then the merge tree            */
     MSORT_OPT_SKIP_TRIVIAL = 2,  /* 1: skip radix passes whose digit is constant (identity permutation)   */
-    MSORT_OPT_HOST_PIPELINE = 3  /* 1 (default): msort_sort_host on ONE GPU overlaps the transfers with the
-                                       sort - the chunk arrives in 4 pieces, each radix sorted while the next
-                                       is in flight, the sorted pieces merge, and the final merge runs in
-                                       slices, each copied back while the next one merges (chunks of at
-                                       least 2^20 keys); 0: H2D, sort, D2H one after the other           */
+    MSORT_OPT_HOST_PIPELINE = 3  /* 1 (default): host sorts overlap the transfers with the sort (chunks of
+                                       at least 2^20 keys) - the chunk arrives in 4 pieces, each radix sorted
+                                       while the next is in flight, and the sorted pieces merge.  One GPU
+                                       (msort_sort_host, g = 1): the final merge runs in slices, each copied
+                                       back while the next one merges.  msort_dist_sort_host: the merged
+                                       chunk enters the merge phase, D2H follows it.  0: H2D, sort, D2H
+                                       one after the other                                                */
 };
 int msort_set_option(msort_ctx* ctx, int option, int64_t value);
 

@@ -1037,16 +1037,22 @@ int msort_sort_device(msort_ctx* ctx, void* const* chunks, uint64_t keys_per_gpu
 // has arrived.  Same result as the sequential path (a sort is unique).
 static constexpr uint64_t kPipeMinKeys = 1ull << 20;
 
-static int sort_host_pipelined(msort_ctx* ctx, char* host, uint64_t n, uint64_t c) {
-    Rank& R = ctx->r[0];
+// S0 + S1-S3 of the pipelined host sort: H2D of `n` keys from `host` into
+// `dst_stage` (c keys, tail padded) in kPieces pieces on the copy stream, each
+// piece radix sorted in place as soon as it has landed (B0 as scratch), pieces
+// 0+1 and 2+3 merged into B0.  Leaves two sorted runs: B0[0, *split) and
+// B0[*split, c).  Records e_h2d0/e_h2d1 (copy stream), e_begin/e_sorted/e_merged.
+static int load_sort_pieces(msort_ctx* ctx, Rank& R, const char* host, uint64_t n, uint64_t c, char* dst_stage,
+                            uint64_t* split) {
     const size_t K = key_bytes(ctx->kt);
-    CUDA_TRY(cudaSetDevice(R.dev));
-    for (bool& b : R.xch_rec) b = false;
-    char* stage = static_cast<char*>(R.stage);
+    char* stage = dst_stage;
     char* b0 = static_cast<char*>(R.buf[0]);
     auto cut = [&](uint64_t num, uint64_t den) { return c * num / den / 1024 * 1024; };
     const uint64_t pb[kPieces + 1] = {0, cut(3, 8), cut(6, 8), cut(15, 16), c};
-    // S0: every piece's H2D (and the tail padding, reading Q3) on the copy stream
+    // S0: every piece's H2D (and the tail padding, reading Q3) on the copy stream,
+    // ordered after the compute stream's earlier work (the staging buffer's last reader)
+    CUDA_TRY(cudaEventRecord(R.e_merged, R.st));
+    CUDA_TRY(cudaStreamWaitEvent(R.cst, R.e_merged, 0));
     CUDA_TRY(cudaEventRecord(R.e_h2d0, R.cst));
     for (int i = 0; i < kPieces; ++i) {
         const uint64_t lo = std::min(pb[i], n), hi = std::min(pb[i + 1], n);
@@ -1075,11 +1081,24 @@ static int sort_host_pipelined(msort_ctx* ctx, char* host, uint64_t n, uint64_t 
         if (i == kPieces - 1) CUDA_TRY(cudaEventRecord(R.e_sorted, R.st));
     }
     CUDA_TRY(cudaEventRecord(R.e_merged, R.st));
+    *split = pb[2];
+    return MSORT_OK;
+}
+
+static int sort_host_pipelined(msort_ctx* ctx, char* host, uint64_t n, uint64_t c) {
+    Rank& R = ctx->r[0];
+    const size_t K = key_bytes(ctx->kt);
+    CUDA_TRY(cudaSetDevice(R.dev));
+    for (bool& b : R.xch_rec) b = false;
+    char* stage = static_cast<char*>(R.stage);
+    char* b0 = static_cast<char*>(R.buf[0]);
+    uint64_t split = 0;
+    MSORT_TRY(load_sort_pieces(ctx, R, host, n, c, stage, &split));
     // S8 overlapped with the final merge: slice co-ranks, then merge + D2H per slice
     const char* A = b0;
-    const uint64_t al = pb[2];
-    const char* B = b0 + pb[2] * K;
-    const uint64_t bl = c - pb[2];
+    const uint64_t al = split;
+    const char* B = b0 + split * K;
+    const uint64_t bl = c - split;
     // co-ranks at multiples of c/64; slices end at 1/64, 1/16, 1/4 and all of
     // the chunk: each copy (PCIe) outlasts the next slice's merge (HBM), so the
     // copies run back to back and only the first, small merge is exposed
@@ -1352,7 +1371,8 @@ static int dist_barrier(msort_ctx* ctx) {
     return MSORT_OK;
 }
 
-static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream, bool keep_timings);
+static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream, bool keep_timings,
+                          const char* host = nullptr);
 
 int msort_dist_sort(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream) {
     return dist_sort_impl(ctx, d_chunk, c, stream, false);
@@ -1367,10 +1387,15 @@ int msort_dist_sort_host(msort_ctx* ctx, void* host_keys, uint64_t c) {
     CUDA_TRY(cudaSetDevice(R.dev));
     reset_timings(ctx, c);
     const size_t K = key_bytes(ctx->kt);
-    CUDA_TRY(cudaEventRecord(R.e_h2d0, R.st));
-    if (c) CUDA_TRY(cudaMemcpyAsync(R.stage, host_keys, c * K, cudaMemcpyHostToDevice, R.st));
-    CUDA_TRY(cudaEventRecord(R.e_h2d1, R.st));
-    MSORT_TRY(dist_sort_impl(ctx, R.stage, c, R.st, true));
+    if (ctx->host_pipeline && c >= kPipeMinKeys) {
+        // pipelined S0 (MSORT_OPT_HOST_PIPELINE): H2D pieces sorted as they land
+        MSORT_TRY(dist_sort_impl(ctx, R.stage, c, R.st, true, static_cast<const char*>(host_keys)));
+    } else {
+        CUDA_TRY(cudaEventRecord(R.e_h2d0, R.st));
+        if (c) CUDA_TRY(cudaMemcpyAsync(R.stage, host_keys, c * K, cudaMemcpyHostToDevice, R.st));
+        CUDA_TRY(cudaEventRecord(R.e_h2d1, R.st));
+        MSORT_TRY(dist_sort_impl(ctx, R.stage, c, R.st, true));
+    }
     CUDA_TRY(cudaEventRecord(R.e_d2h0, R.st));
     if (c) CUDA_TRY(cudaMemcpyAsync(host_keys, R.stage, c * K, cudaMemcpyDeviceToHost, R.st));
     CUDA_TRY(cudaEventRecord(R.e_d2h1, R.st));
@@ -1381,7 +1406,8 @@ int msort_dist_sort_host(msort_ctx* ctx, void* host_keys, uint64_t c) {
     return MSORT_OK;
 }
 
-static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream, bool keep_timings) {
+static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream, bool keep_timings,
+                          const char* host) {
     if (!ctx || !ctx->dist || !ctx->imported) return set_error(MSORT_ERR_INVALID_ARGUMENT, "dist ctx not imported");
     if (c && !d_chunk) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL chunk");
     MSORT_TRY(check_c(ctx, c));
@@ -1397,17 +1423,22 @@ static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* strea
     R.user = d_chunk;
     CUDA_TRY(cudaEventRecord(R.e_begin, R.st));
     if (c == 0) return MSORT_OK;
-    // S1-S3
-    MSORT_TRY(radix_begin(ctx, R, d_chunk, c));
-    if (ctx->skip_trivial) CUDA_TRY(cudaStreamSynchronize(R.st));
+    // S1-S3 (host != NULL: S0 too, pipelined - the chunk lands from `host` in
+    // pieces, each sorted while the next is in flight, then merged)
     int cur[MSORT_MAX_GPUS];
-    if (g == 1) {
-        MSORT_TRY(radix_passes(ctx, R, d_chunk, d_chunk, R.buf[0], c));
-        for (int q = 0; q < g; ++q) cur[q] = -1;
+    void* sorted_dst = g == 1 ? d_chunk : R.buf[1];
+    if (host) {
+        uint64_t split = 0;
+        MSORT_TRY(load_sort_pieces(ctx, R, host, c, c, static_cast<char*>(d_chunk), &split));
+        const char* b0 = static_cast<const char*>(R.buf[0]);
+        CUDA_TRY(launch_merge(b0, split, b0 + split * key_bytes(ctx->kt), c - split, sorted_dst, ctx->kt, R.mws, R.st,
+                              &ctx->tm.kernel_launches));
     } else {
-        MSORT_TRY(radix_passes(ctx, R, d_chunk, R.buf[1], R.buf[0], c));
-        for (int q = 0; q < g; ++q) cur[q] = 1;
+        MSORT_TRY(radix_begin(ctx, R, d_chunk, c));
+        if (ctx->skip_trivial) CUDA_TRY(cudaStreamSynchronize(R.st));
+        MSORT_TRY(radix_passes(ctx, R, d_chunk, sorted_dst, R.buf[0], c));
     }
+    for (int q = 0; q < g; ++q) cur[q] = g == 1 ? -1 : 1;
     CUDA_TRY(cudaEventRecord(R.e_sorted, R.st));
     if (g > 1 && ctx->exchange >= 2) {
         // NEXT-1: splitters from every peer's sorted chunk, one pull per peer,

@@ -71,6 +71,10 @@ def _worker(rank, world, port, n, kt, distn, out_dir, host, exchange=0):
     (8, 80_000, "f32", "uniform", True, 2),
     (4, 200_001, "u32", "zipf", False, 3),
     (2, 90_001, "u64", "uniform", True, 3),
+    # chunks of >= 2^20 keys: msort_dist_sort_host takes the pipelined S0 (pieces sorted as they land)
+    (2, 2_500_001, "u32", "uniform", True, 0),
+    (4, 4_400_000, "f32", "uniform", True, 2),
+    (2, 2_200_002, "u32", "zipf", True, 3),
 ])
 def test_dist_sort_matches_oracle(tmp_path, world, n, kt, distn, host, exchange):
     mp.spawn(_worker, args=(world, _free_port(), n, kt, distn, str(tmp_path), host, exchange), nprocs=world,
