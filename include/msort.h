@@ -117,13 +117,17 @@ enum {
                                        3: NEXT-1 with the exchange as separate pulls (every GPU copies its run
                                        from every chunk into a local buffer), then the merge tree            */
     MSORT_OPT_SKIP_TRIVIAL = 2,  /* 1: skip radix passes whose digit is constant (identity permutation)   */
-    MSORT_OPT_HOST_PIPELINE = 3  /* 1 (default): host sorts overlap the transfers with the sort (chunks of
+    MSORT_OPT_HOST_PIPELINE = 3, /* 1 (default): host sorts overlap the transfers with the sort (chunks of
                                        at least 2^20 keys) - the chunk arrives in 4 pieces, each radix sorted
                                        while the next is in flight, and the sorted pieces merge.  One GPU
                                        (msort_sort_host, g = 1): the final merge runs in slices, each copied
                                        back while the next one merges.  msort_dist_sort_host: the merged
                                        chunk enters the merge phase, D2H follows it.  0: H2D, sort, D2H
                                        one after the other                                                */
+    MSORT_OPT_SMALL_GRAPH = 4    /* 1 (default): a one-GPU device sort of <= 2^22 keys repeated on the same
+                                       buffer and size replays the whole radix sort as one CUDA graph
+                                       (captured on the second call; all passes run, no host round trip on
+                                       the histogram); 0: always the launch-by-launch path              */
 };
 int msort_set_option(msort_ctx* ctx, int option, int64_t value);
 

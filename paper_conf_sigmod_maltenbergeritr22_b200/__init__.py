@@ -28,7 +28,7 @@ KEY_BYTES = {0: 4, 1: 8, 2: 4, 3: 8}
 MSORT_MAX_GPUS = 8
 MSORT_MAX_STAGES = 7
 MSORT_DIST_HANDLE_BYTES = 512
-MSORT_OPT_TIMING, MSORT_OPT_EXCHANGE, MSORT_OPT_SKIP_TRIVIAL, MSORT_OPT_HOST_PIPELINE = 0, 1, 2, 3
+MSORT_OPT_TIMING, MSORT_OPT_EXCHANGE, MSORT_OPT_SKIP_TRIVIAL, MSORT_OPT_HOST_PIPELINE, MSORT_OPT_SMALL_GRAPH = 0, 1, 2, 3, 4
 EXCHANGE_FUSED, EXCHANGE_SWAP, EXCHANGE_ALLTOALL, EXCHANGE_ALLTOALL_PULL = 0, 1, 2, 3
 MSORT_PASS_ENCODE_IN, MSORT_PASS_DECODE_OUT = 1, 2
 

@@ -149,6 +149,13 @@ struct Rank {
     cudaEvent_t e_piece[kPieces] = {};
     cudaEvent_t e_slice[kSlices] = {};
     cudaEvent_t e_merged = nullptr;
+    // small one-GPU sorts (<= kGraphMaxKeys): the whole radix sort as one CUDA
+    // graph, captured when the same (buffer, size) is sorted a second time
+    cudaGraphExec_t small_exec = nullptr;
+    const void* small_user = nullptr;
+    uint64_t small_c = 0;
+    int small_timing = -1;
+    bool small_seen = false;
     cudaEvent_t e_sync[MSORT_MAX_STAGES + 1] = {};
     cudaEvent_t e_stage[MSORT_MAX_STAGES][2] = {};
     cudaEvent_t e_xch[MSORT_MAX_STAGES][2] = {};
@@ -193,6 +200,7 @@ struct msort_ctx {
     int exchange = 0;
     int skip_trivial = 1;
     int host_pipeline = 1;
+    int small_graph = 1;
     msort_timings tm{};
 };
 
@@ -267,6 +275,7 @@ void free_rank(Rank& R) {
     for (auto e : R.e_slice)
         if (e) cudaEventDestroy(e);
     if (R.e_merged) cudaEventDestroy(R.e_merged);
+    if (R.small_exec) cudaGraphExecDestroy(R.small_exec);
     if (R.cst) {
         cudaStreamSynchronize(R.cst);
         cudaStreamDestroy(R.cst);
@@ -612,8 +621,86 @@ int alltoall_local(msort_ctx* ctx, uint64_t c) {
     return MSORT_OK;
 }
 
+// Small sorts on one GPU (2^20 keys are L2-resident, so the
+// sort is launch- and latency-bound).  The sequence of msort_radix_sort -
+// workspace zeroing, histogram, scan, all P passes (a constant digit's pass is
+// an identity permutation: no host round trip on the trivial flags; default
+// ranking without the skew hints) - captured once as a CUDA graph and replayed
+// while the caller sorts the same buffer and size again.  The first call with a
+// new (buffer, size) runs the normal path and only remembers it.
+static constexpr uint64_t kGraphMaxKeys = 1ull << 22;
+
+int capture_small(msort_ctx* ctx, Rank& R, uint64_t c) {
+    const int P = num_passes(ctx->kt);
+    if (R.small_exec) {
+        cudaGraphExecDestroy(R.small_exec);
+        R.small_exec = nullptr;
+    }
+    cudaGraph_t graph = nullptr;
+    CUDA_TRY(cudaStreamBeginCapture(R.st, cudaStreamCaptureModeThreadLocal));
+    // timing events inside the graph are external records (recorded on every replay)
+    auto rec = [&](cudaEvent_t e) { return cudaEventRecordWithFlags(e, R.st, cudaEventRecordExternal); };
+    auto body = [&]() -> int {
+        RadixWs ws = radix_ws_layout(R.rws, c, ctx->kt);
+        ws.epoch = 0;  // every replay zeroes the (small) workspace: status tags repeat
+        CUDA_TRY(radix_prologue(R.user, c, ctx->kt, ws, R.st));
+        if (ctx->timing) CUDA_TRY(rec(R.e_hist));
+        for (int p = 0; p < P; ++p) {
+            const void* in = (p % 2 == 0) ? R.user : R.buf[0];
+            void* out = (p % 2 == 0) ? R.buf[0] : R.user;
+            const int flags = (p == 0 ? 1 : 0) | (p == P - 1 ? 2 : 0) | ((p == 0 || atomic_rank_ok()) ? 4 : 0);
+            if (ctx->timing) CUDA_TRY(rec(R.e_pass[p][0]));
+            CUDA_TRY(launch_onesweep(in, out, c, ctx->kt, p, flags, ws, ws.base + p * 256, R.st));
+            if (ctx->timing) CUDA_TRY(rec(R.e_pass[p][1]));
+        }
+        return MSORT_OK;
+    };
+    const int st = body();
+    const cudaError_t ce = cudaStreamEndCapture(R.st, &graph);
+    if (st != MSORT_OK) {
+        if (graph) cudaGraphDestroy(graph);
+        return st;
+    }
+    CUDA_TRY(ce);
+    const cudaError_t ie = cudaGraphInstantiate(&R.small_exec, graph, 0);
+    cudaGraphDestroy(graph);
+    CUDA_TRY(ie);
+    R.small_user = R.user;
+    R.small_c = c;
+    R.small_timing = ctx->timing;
+    return MSORT_OK;
+}
+
+// true if the sort ran as a graph replay
+int sort_small_graph(msort_ctx* ctx, Rank& R, uint64_t c, bool* done) {
+    *done = false;
+    const bool same = R.small_user == R.user && R.small_c == c;
+    if (!same) {  // remember; capture if it comes again
+        if (R.small_exec) cudaGraphExecDestroy(R.small_exec);
+        R.small_exec = nullptr;
+        R.small_user = R.user;
+        R.small_c = c;
+        return MSORT_OK;
+    }
+    if (!R.small_exec || R.small_timing != ctx->timing) MSORT_TRY(capture_small(ctx, R, c));
+    CUDA_TRY(cudaEventRecord(R.e_begin, R.st));
+    CUDA_TRY(cudaGraphLaunch(R.small_exec, R.st));
+    CUDA_TRY(cudaEventRecord(R.e_sorted, R.st));
+    CUDA_TRY(cudaEventRecord(R.e_end, R.st));
+    ctx->tm.kernel_launches += 2 + num_passes(ctx->kt);
+    R.passes_run = num_passes(ctx->kt);
+    R.cur = -1;
+    *done = true;
+    return MSORT_OK;
+}
+
 int sort_device_local(msort_ctx* ctx, uint64_t c) {
     const int g = ctx->g;
+    if (g == 1 && c <= kGraphMaxKeys && ctx->small_graph) {
+        bool done = false;
+        MSORT_TRY(sort_small_graph(ctx, ctx->r[0], c, &done));
+        if (done) return MSORT_OK;
+    }
     std::vector<int> labels;
     stage_labels(g, labels);
     for (int i = 0; i < g; ++i) {
@@ -949,6 +1036,7 @@ int msort_set_option(msort_ctx* ctx, int option, int64_t value) {
         case MSORT_OPT_TIMING: ctx->timing = value ? 1 : 0; return MSORT_OK;
         case MSORT_OPT_SKIP_TRIVIAL: ctx->skip_trivial = value ? 1 : 0; return MSORT_OK;
         case MSORT_OPT_HOST_PIPELINE: ctx->host_pipeline = value ? 1 : 0; return MSORT_OK;
+        case MSORT_OPT_SMALL_GRAPH: ctx->small_graph = value ? 1 : 0; return MSORT_OK;
         case MSORT_OPT_EXCHANGE:
             if (value < 0 || value > 3) return set_error(MSORT_ERR_INVALID_ARGUMENT, "exchange mode 0, 1, 2 or 3");
             if (value == 1)

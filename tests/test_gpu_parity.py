@@ -307,6 +307,36 @@ def test_sort_host_pipelined(ms, kt, dist, n, pipeline):
     assert t["total_ms"] > 0 and t["h2d_ms"] > 0 and t["d2h_ms"] > 0
 
 
+def _shaped(n, kt, dist, seed):
+    """distribution shapes for every key type (u64 / f32 from the u32 shapes' bits)"""
+    if kt in ("u32",) or dist == "uniform":
+        return mi.np_generate(n, kt, dist, seed=seed)
+    a = mi.np_generate(n, "u32", dist, seed=seed)
+    return {"u64": a.astype(np.uint64) * np.uint64(0x10001), "f32": a.view(np.float32),
+            "f64": (a.astype(np.uint64) << np.uint64(32)).view(np.float64)}[kt]
+
+
+@pytest.mark.parametrize("kt", ["u32", "u64", "f32", "f64"])
+def test_small_sort_graph_replay(ms, kt):
+    """Repeated one-GPU sorts of one buffer (MSORT_OPT_SMALL_GRAPH: the second call
+    captures the radix sort as a CUDA graph, later calls replay it) on new data each
+    time, skewed and sorted shapes included, then a new size (re-capture): every
+    result equals the oracle (§8(c))."""
+    K = mi.KEY_BYTES[kt]
+    for n in ((1 << 20) + 5, 300_001):
+        buf = torch.empty(n * K, dtype=torch.uint8, device="cuda")
+        ctx = ms.Context(1, n, kt, device_ids=[0])
+        for trial, dist in enumerate(["uniform", "zipf", "uniform", "reverse", "sorted", "uniform"]):
+            a = _shaped(n, kt, dist, seed=trial)
+            buf.copy_(torch.from_numpy(a.view(np.uint8).copy()))
+            ctx.sort_device([ms.tensor_ptr(buf)], n)
+            got = buf.cpu().numpy().view(codec.UINT[kt])
+            assert got.tobytes() == bits(sort.oracle_sort(a, kt), kt).tobytes(), (n, trial, dist)
+        t = ctx.timings()
+        assert t["passes_run"] == radix.num_passes(kt)
+        ctx.close()
+
+
 def test_msort_sort_host_pointer(ms):
     n = 100003
     a = mi.np_generate(n, "f32", "uniform", seed=9)
