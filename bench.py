@@ -57,9 +57,12 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--seed", type=int, default=1)
-    ap.add_argument("--exchange", type=int, default=0,
+    ap.add_argument("--exchange", type=int, default=None,
                     help="merge phase for N>1: 0 the paper's Alg.2 with fused exchange+merge, 1 Alg.2 swap then "
-                         "merge (single process only), 2 NEXT-1 single all-to-all fused into the merge, 3 NEXT-1 pull then merge")
+                         "merge (single process only), 2 (default for N>1) NEXT-1 - the paper's future work for "
+                         "NVSwitch systems, P:3416-3424 - single all-to-all fused into the merge, 3 NEXT-1 pull then "
+                         "merge. With 2 or 3, Alg.2 (0) is timed too and reported as `alg2`")
+    ap.add_argument("--no-alg2", action="store_true", help="N>1: skip the Alg.2 comparison timing")
     ap.add_argument("--het", action="store_true", help="also time the HET-sort baseline (GPU chunk sort + CPU merge)")
     ap.add_argument("--het-chunks", type=int, default=8)
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -267,6 +270,8 @@ def main():
         from paper_conf_sigmod_maltenbergeritr22_b200 import dist as mdist
         ctx = mdist.dist_context(rank, g, local, c, kt)
         sort_dev = lambda: ctx.sort(ms.tensor_ptr(work), c, stream=stream)  # noqa: E731
+    if args.exchange is None:
+        args.exchange = 2 if g > 1 else 0
     if g > 1:
         if args.exchange == 1:
             raise SystemExit("--exchange 1 (swap then merge) is a single-process option")
@@ -317,6 +322,34 @@ def main():
         tot = float(tt.item())
     ms_per_step = tot / args.steps
     value = n / (ms_per_step / 1e3)
+
+    # --- N>1 with NEXT-1: the paper's own merge phase (Alg.2) timed the same way, as context
+    alg2 = None
+    if g > 1 and args.exchange in (2, 3) and not args.no_alg2:
+        ctx.set_option(ms.MSORT_OPT_EXCHANGE, 0)
+        for _ in range(2):
+            with torch.cuda.stream(stream):
+                work.copy_(pristine)
+            sort_dev()
+        barrier()
+        ev2 = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        for i in range(args.steps):
+            with torch.cuda.stream(stream):
+                work.copy_(pristine)
+                ev2[i][0].record(stream)
+            sort_dev()
+            with torch.cuda.stream(stream):
+                ev2[i][1].record(stream)
+        barrier()
+        t2 = sum(a.elapsed_time(b) for a, b in ev2)
+        tt = torch.tensor([t2], dtype=torch.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms2 = float(tt.item()) / args.steps
+        at = ctx.timings()
+        alg2 = {"value": n / (ms2 / 1e3), "unit": "keys/s", "ms_per_step": ms2,
+                "exchange": "Alg.2 (paper P:1763-1854), fused peer-read merge", "merge_phase_ms": at["merge_ms"],
+                "stage_label": at["stage_label"], "stage_max_x": at["stage_max_x"]}
+        ctx.set_option(ms.MSORT_OPT_EXCHANGE, args.exchange)
 
     # --- roofline of the dominant kernel (onesweep pass)
     peak, peak_src = hbm_peak()
@@ -419,6 +452,7 @@ def main():
                                                   "stage_exchange_ms")} if stage_info and g > 1 else None,
             "paper_context": PAPER_CONTEXT,
             "het_baseline": het,
+            "alg2": alg2,
         }
         print(json.dumps(out))
     if dist:
