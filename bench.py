@@ -3,8 +3,11 @@
 
 Workload (BASELINE.json configs[2], paper Fig.1 shape): 4e9 uniform uint32 keys
 (16 GB), sorted on N = 1/2/4/8 GPUs (strong scaling: the total is fixed).  A
-"step" is one whole sort: per-GPU radix sort (S1-S3) and, for N > 1, the g-1
-merge stages (S4-S7).
+"step" is one whole sort: per-GPU radix sort (S1-S3) and, for N > 1, the merge
+phase: by default NEXT-1, the paper's future work for NVSwitch systems
+(one all-to-all exchange fused into a local merge tree), with the
+paper's own g-1 merge stages (Alg.2, S4-S7) timed beside it as `alg2`
+(`--exchange 0` makes Alg.2 the measured path).
 
   value  device-resident keys/s: chunks already in HBM; CUDA events on the
          stream the sort is ordered on, max over ranks; the input is restored
@@ -12,7 +15,8 @@ merge stages (S4-S7).
          16 GB >> 126 MB L2, so no L2 flush is needed)
   e2e    the same metric through the public host-pointer API (msort_sort_host /
          msort_dist_sort_host): pinned host keys -> H2D -> sort -> D2H, timed
-         per call
+         per call; N = 1: the pipelined path (transfers overlapped with the
+         sort), the sequential one interleaved with it as `e2e.sequential`
   roofline  dominant kernel = the onesweep pass (S3): algorithmic bytes
          2*K*c per launch / mean launch time (library CUDA events around each
          launch) vs MEASURED_PEAKS.json hbm_gbs
