@@ -390,6 +390,13 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     if (Cfg::kAnyOr) {
         for (int i = tid; i < WARPS * kRadix; i += THREADS) (&s_match[0][0])[i] = 0;
     }
+    // per-warp digit counters start at zero; each tile re-zeroes them during its
+    // scatter (they are dead after the ranking), so no barrier of its own
+    auto zero_counts = [&]() {
+        uint4* z = reinterpret_cast<uint4*>(&s_cnt[0][0]);
+        for (int i = tid; i < WARPS * kRadix / 4; i += THREADS) z[i] = make_uint4(0, 0, 0, 0);
+    };
+    zero_counts();
     if (tid == 0) {
         // Tile ids in arrival order: every lower tile is already held by a
         // running block, so the look-back below always makes progress.
@@ -408,12 +415,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
 #pragma unroll
             for (int i = 0; i < ITEMS; ++i) keys[i] = encode<U, FLOAT>(keys[i]);
         }
-        {
-            uint4* z = reinterpret_cast<uint4*>(&s_cnt[0][0]);
-            for (int i = tid; i < WARPS * kRadix / 4; i += THREADS) z[i] = make_uint4(0, 0, 0, 0);
-        }
-        __syncthreads();  // s_cnt zeroed
-
+        // (s_cnt was zeroed during the previous tile's scatter, or before the loop)
 
         // --- early counts: per-warp digit histogram (fire-and-forget smem adds).
         // kCountRank (atomic-ranked passes): the count's returned value is the
@@ -571,6 +573,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
                 out[dst] = DEC_OUT ? decode<U, FLOAT>(k) : k;
             }
         }
+        zero_counts();  // for the next tile (ordered before its count atomics by the barrier below)
         __syncthreads();
         tile = Cfg::kPrefetch ? next_tile : s_next;
     }

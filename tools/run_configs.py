@@ -19,15 +19,21 @@ CONFIGS = [  # (BASELINE.json configs index, n, g, key type, distribution, excha
     (1, 1 << 28, 2, "u32", "uniform", 0),
     (2, 4_000_000_000, 1, "u32", "uniform", 0),
     (2, 4_000_000_000, 2, "u32", "uniform", 0),
+    (2, 4_000_000_000, 2, "u32", "uniform", 2),
     (2, 4_000_000_000, 4, "u32", "uniform", 0),
+    (2, 4_000_000_000, 4, "u32", "uniform", 2),
     (2, 4_000_000_000, 8, "u32", "uniform", 0),
     (2, 4_000_000_000, 8, "u32", "uniform", 2),
     (3, 2_000_000_000, 8, "u32", "zipf", 0),
     (3, 2_000_000_000, 8, "u32", "sorted", 0),
     (3, 2_000_000_000, 8, "u32", "reverse", 0),
     (3, 2_000_000_000, 8, "u32", "nearly", 0),
+    (3, 2_000_000_000, 8, "u32", "zipf", 2),
+    (3, 2_000_000_000, 8, "u32", "reverse", 2),
     (4, 2_000_000_000, 8, "u64", "uniform", 0),
+    (4, 2_000_000_000, 8, "u64", "uniform", 2),
     (4, 2_000_000_000, 8, "f32", "uniform", 0),
+    (4, 2_000_000_000, 8, "f32", "uniform", 2),
 ]
 only = os.environ.get("CONFIGS")
 for idx, n, g, kt, dist, ex in CONFIGS:
