@@ -202,9 +202,10 @@ struct OsCfg {
     static constexpr uint32_t kTile = uint32_t(THREADS_) * ITEMS_;
     static constexpr bool kAnyOr = (BALLOT_MASK_ & ((ITEMS_ >= 32 ? 0u : (1u << ITEMS_)) - 1u)) !=
                                    ((ITEMS_ >= 32 ? 0u : (1u << ITEMS_)) - 1u);
-    template <typename U>
+    // (the atomicOr peer masks exist only in the peer-match ranking, STABLE)
+    template <typename U, bool STABLE = true>
     static constexpr size_t smem_bytes() {
-        return size_t(kTile) * sizeof(U) + size_t(kWarps) * kRadix * 4 * (kAnyOr ? 2 : 1);
+        return size_t(kTile) * sizeof(U) + size_t(kWarps) * kRadix * 4 * (kAnyOr && STABLE ? 2 : 1);
     }
 };
 
@@ -387,7 +388,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
         return excl;
     };
 
-    if (Cfg::kAnyOr) {
+    if (Cfg::kAnyOr && STABLE) {  // (atomic-ranked kernels have no peer-mask array)
         for (int i = tid; i < WARPS * kRadix; i += THREADS) (&s_match[0][0])[i] = 0;
     }
     // per-warp digit counters start at zero; each tile re-zeroes them during its
@@ -674,7 +675,7 @@ __global__ void __launch_bounds__(256) rank_probe_kernel(uint32_t seed, uint32_t
 template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg, bool STABLE>
 cudaError_t launch_onesweep_c(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
                               const uint32_t* base_row, uint32_t tag, cudaStream_t st, uint32_t hot, bool hot_on) {
-    const size_t smem = Cfg::template smem_bytes<U>();
+    const size_t smem = Cfg::template smem_bytes<U, STABLE>();
     auto kern = onesweep_kernel<U, FLOAT, ENC_IN, DEC_OUT, Cfg, STABLE>;
     // per-device attribute: set on every launch (cheap, and correct when one
     // process drives several GPUs)

@@ -108,6 +108,23 @@ def test_config3_4e9_u32_one_gpu():
     _check(chunks, n, "u32", "uniform", 1)
 
 
+def test_max_chunk_u32_one_gpu():
+    """The largest chunk the 32-bit per-chunk indexing contract allows (include/msort.h: keys per GPU < 2^32,
+    rounded to a multiple of 4, reading Q3): n = 2^32 - 4 uint32 keys on one GPU, sorted device-resident and
+    checked like configs[2]; one key more per GPU is refused with MSORT_ERR_INVALID_ARGUMENT, not truncated."""
+    import paper_conf_sigmod_maltenbergeritr22_b200 as ms
+    n = (1 << 32) - 4
+    chunks, c = _gen_chunks(n, 1, "u32", "uniform", 3)
+    ctx = ms.Context(1, n, "u32", device_ids=[0])
+    ctx.sort_device([ms.tensor_ptr(chunks[0])], c)
+    torch.cuda.synchronize()
+    ctx.close()
+    _check(chunks, n, "u32", "uniform", 3)
+    with pytest.raises(ms.MsortError) as e:
+        ms.Context(1, n + 1, "u32", device_ids=[0])
+    assert "INVALID_ARGUMENT" in str(e.value)
+
+
 def test_config3_4e9_u32_one_gpu_end_to_end():
     """configs[2] end to end (bench.py's e2e call): pinned host keys -> msort_sort_host
     (pipelined transfers, MSORT_OPT_HOST_PIPELINE default) -> host; checked on the GPU."""
