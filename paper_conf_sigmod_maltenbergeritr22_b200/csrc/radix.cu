@@ -184,28 +184,6 @@ __device__ __forceinline__ uint32_t ballot_match8(uint32_t d) {
     return peers;
 }
 
-#ifndef MSORT_LDHINT
-#define MSORT_LDHINT 0  // tile loads: 0 = ld.global.cs (streaming), 1 = L1::no_allocate, 2 = ld.global.nc
-#endif
-template <typename U>
-__device__ __forceinline__ U load_key(const U* p) {
-#if MSORT_LDHINT == 1
-    if constexpr (sizeof(U) == 4) {
-        uint32_t v;
-        asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(v) : "l"(p));
-        return U(v);
-    } else {
-        unsigned long long v;
-        asm volatile("ld.global.nc.L1::no_allocate.u64 %0, [%1];" : "=l"(v) : "l"(p));
-        return U(v);
-    }
-#elif MSORT_LDHINT == 2
-    return __ldg(p);
-#else
-    return __ldcs(p);
-#endif
-}
-
 // THREADS x ITEMS keys per tile; bit i of BALLOT_MASK: item i ranks with the
 // ballot match (else smem atomicOr); MINB blocks per SM for __launch_bounds__.
 template <int THREADS_, int ITEMS_, uint32_t BALLOT_MASK_, int MINB_, bool PF_, int LB_ = 4, bool ELB_ = false,
@@ -281,7 +259,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
         const U* src = in + tb + wofs;
         if (tb + TILE <= n) {
 #pragma unroll
-            for (int i = 0; i < ITEMS; ++i) keys[i] = load_key(src + i * 32);
+            for (int i = 0; i < ITEMS; ++i) keys[i] = __ldcs(src + i * 32);
         } else {
 #pragma unroll
             for (int i = 0; i < ITEMS; ++i) {
