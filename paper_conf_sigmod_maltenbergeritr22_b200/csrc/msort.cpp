@@ -57,6 +57,7 @@ int cuda_status(cudaError_t e) {
     do {                                                                                                \
         cudaError_t e_ = (expr);                                                                        \
         if (e_ != cudaSuccess) {                                                                        \
+            cudaGetLastError(); /* clear a non-sticky error (e.g. a failed allocation) for later calls */ \
             return set_error(cuda_status(e_), std::string(#expr) + " -> " + cudaGetErrorString(e_) +   \
                                                   " (" + __FILE__ + ":" + std::to_string(__LINE__) + ")"); \
         }                                                                                               \

@@ -245,7 +245,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     __shared__ uint32_t s_next;
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const uint32_t ntiles = (n + TILE - 1) / TILE;
+    const uint32_t ntiles = uint32_t((uint64_t(n) + TILE - 1) / TILE);  // (64-bit: n may be 2^32 - 4)
     const uint32_t lt = lanemask_lt();
     const uint32_t wofs = uint32_t(warp) * 32 * ITEMS + lane;
 

@@ -355,6 +355,23 @@ def test_errors(ms):
     ms.msort_sort(0, 0, "u32", 1)   # n = 0 is a no-op
 
 
+def test_out_of_memory_is_reported_and_recoverable(ms):
+    """A context larger than HBM (8 virtual ranks x (2^32 - 4) u64 keys: 3 chunk buffers of 32 GB each per
+    rank) fails with MSORT_ERR_OUT_OF_MEMORY (include/msort.h: no CPU fallback) and leaves the device usable:
+    what it had allocated is freed and the next context sorts correctly."""
+    n = 8 * ((1 << 32) - 4)
+    with pytest.raises(ms.MsortError) as e:
+        ms.Context(8, n, "u64", device_ids=[0] * 8)
+    assert "OUT_OF_MEMORY" in str(e.value)
+    a = mi.np_generate(100_003, "u64", "uniform", seed=8)
+    d = dev_keys(a)
+    ctx = ms.Context(1, a.size, "u64", device_ids=[0])
+    ctx.sort_device([ms.tensor_ptr(d)], a.size)
+    torch.cuda.synchronize()
+    ctx.close()
+    assert np.array_equal(host_keys(d, "u64"), sort.oracle_sort(a, "u64"))
+
+
 # ---------------------------------------------------------------------------
 # NEXT-1: single all-to-all exchange (MSORT_OPT_EXCHANGE = 2 fused, 3 pull-then-merge)
 # ---------------------------------------------------------------------------
