@@ -7,6 +7,14 @@ import torch
 import msort_inputs as mi
 import paper_conf_sigmod_maltenbergeritr22_b200 as ms
 n = int(float(sys.argv[1])); kt = sys.argv[2]; reps = int(sys.argv[3]) if len(sys.argv) > 3 else 3
+if len(sys.argv) > 4 and sys.argv[4] == "numa":  # pin to the GPU's NUMA-local CPUs before any host allocation
+    import pynvml
+    pynvml.nvmlInit()
+    h = pynvml.nvmlDeviceGetHandleByIndex(0)
+    words = pynvml.nvmlDeviceGetCpuAffinity(h, (os.cpu_count() + 63) // 64)
+    cpus = {w * 64 + b for w, m in enumerate(words) for b in range(64) if (m >> b) & 1}
+    print(json.dumps({"affinity_before": len(os.sched_getaffinity(0)), "gpu_local_cpus": len(cpus)}))
+    os.sched_setaffinity(0, cpus & os.sched_getaffinity(0) or cpus)
 src = torch.empty(n, dtype=mi.torch_dtype(kt), device="cuda")
 mi.t_generate_into(src, n, kt, "uniform", seed=1, block=1 << 27)
 pristine = src.cpu()
