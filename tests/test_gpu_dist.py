@@ -86,3 +86,79 @@ def test_dist_sort_matches_oracle(tmp_path, world, n, kt, distn, host, exchange)
     assert np.array_equal(out, codec.bits_of(sort.oracle_sort(a, kt), kt))
     labels = eval((tmp_path / "t0.txt").read_text())
     assert len(labels) == (world - 1 if exchange < 2 else 1)
+
+
+def _worker_big(rank, world, port, n, kt, distn, exchange, out_dir):
+    """Full-size rank: this rank's chunk of the seeded workload generated on the GPU, sorted through
+    msort_dist_sort, summarised by properties that hold at any size (oracle.checks)."""
+    import json
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    os.environ.setdefault("MSORT_BARRIER_TIMEOUT_S", "300")
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import paper_conf_sigmod_maltenbergeritr22_b200 as m
+    from paper_conf_sigmod_maltenbergeritr22_b200 import dist as md
+    from oracle import checks
+    ch = md.chunking(n, world)
+    c, v = ch.c, ch.valid(rank)
+    t = torch.empty(c, dtype=mi.torch_dtype(kt), device="cuda")
+    mi.t_generate_into(t[:v], n, kt, distn, seed=9, start=ch.offset(rank), block=1 << 27)
+    if v < c:  # reading Q3 padding (the largest key under T), as a signed bit pattern of the key width
+        signed = np.int32 if mi.KEY_BYTES[kt] == 4 else np.int64
+        pad = int(np.array([md.PAD_BITS[kt]], dtype=codec.UINT[kt]).view(signed)[0])
+        t.view(torch.int32 if mi.KEY_BYTES[kt] == 4 else torch.int64)[v:] = pad
+    blk = 1 << 26
+
+    def fp(x, lim):
+        f = [0, 0, 0]
+        for off in range(0, lim, blk):
+            a, b, cc = checks.fingerprint(x[off:min(off + blk, lim)].cpu().numpy(), kt)
+            f = [f[0] + a, (f[1] + b) % (1 << 64), f[2] ^ cc]
+        return f
+    fp_in = fp(t, v)
+    ctx = md.dist_context(rank, world, 0, c, kt)
+    ctx.set_option(m.MSORT_OPT_EXCHANGE, exchange)
+    ctx.sort(m.tensor_ptr(t), c)
+    torch.cuda.synchronize()
+    # pads sort to the global end: the valid outputs are the first n of the concatenation
+    keep = max(0, min(c, n - rank * c))
+    ok, first, last = True, None, None
+    for off in range(0, keep, blk):
+        codes = codec.encode(t[off:min(off + blk, keep)].cpu().numpy(), kt)
+        ok &= checks.is_sorted_codes(codes)
+        ok &= last is None or int(last) <= int(codes[0])
+        first = int(codes[0]) if first is None else first
+        last = int(codes[-1])
+    res = {"fp_in": fp_in, "fp_out": fp(t, keep), "sorted": bool(ok), "first": first, "last": last}
+    with open(os.path.join(out_dir, f"big{rank}.json"), "w") as f:
+        json.dump(res, f)
+    ctx.close()
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,n,kt,distn,exchange", [
+    (4, 1_000_000_003, "u32", "uniform", 2),   # bench.py's N > 1 path (NEXT-1 fused), ranks sharing one GPU
+    (2, 1_000_000_000, "u32", "zipf", 0),      # the paper's Alg.2 with the fused peer-read merge
+])
+def test_dist_sort_full_size(tmp_path, world, n, kt, distn, exchange):
+    """One process per rank at full size: every rank's output non-decreasing, rank boundaries ordered, and the
+    union a permutation of the input (fingerprints) - together equality with the unique sorted result
+    (oracle/checks.py)."""
+    import json
+    mp.spawn(_worker_big, args=(world, _free_port(), n, kt, distn, exchange, str(tmp_path)), nprocs=world, join=True)
+    rs = [json.loads((tmp_path / f"big{r}.json").read_text()) for r in range(world)]
+    assert all(r["sorted"] for r in rs)
+    for a, b in zip(rs, rs[1:]):
+        if a["last"] is not None and b["first"] is not None:
+            assert a["last"] <= b["first"]
+
+    def tot(k):
+        f = [0, 0, 0]
+        for r in rs:
+            f = [f[0] + r[k][0], (f[1] + r[k][1]) % (1 << 64), f[2] ^ r[k][2]]
+        return f
+    assert tot("fp_in") == tot("fp_out") and tot("fp_in")[0] == n

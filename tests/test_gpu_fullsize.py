@@ -150,6 +150,11 @@ def test_config3_4e9_u32_one_gpu_end_to_end():
     (2_000_000_000, 8, "f32", "uniform", 0),     # configs[4] float keys
     (2_000_000_000, 8, "u64", "uniform", 0),     # configs[4] 64-bit keys
     (2_000_000_000, 8, "u32", "zipf", 2),        # NEXT-1 (fused all-to-all) at full size
+    (4_000_000_000, 8, "u32", "uniform", 2),     # configs[2] as bench.py measures it at N = 8 (NEXT-1 default)
+    (4_000_000_000, 4, "u32", "uniform", 2),     # ... at N = 4
+    (1 << 28, 2, "u32", "uniform", 2),           # configs[1] with NEXT-1
+    (2_000_000_000, 8, "u64", "uniform", 2),     # configs[4] 64-bit keys, NEXT-1
+    (2_000_000_000, 8, "f32", "uniform", 3),     # configs[4] float keys, NEXT-1 pull-then-merge
 ])
 def test_p2p_virtual_full_size(n, g, kt, dist, exchange):
     import paper_conf_sigmod_maltenbergeritr22_b200 as ms
