@@ -588,11 +588,11 @@ using Cfg32_0 = OsCfg<256, 28, 0x5555555u, 4, true, 2, false, false, 32>;  // 71
                                                                            // look-back window 2, groups of 32 (best)
 using Cfg32_1 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 0>;   // tile-by-tile look-back only
 using Cfg32_2 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 16>;  // look-back groups of 16
-using Cfg32_3 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 64>;  // look-back groups of 64
+using Cfg32_3 = OsCfg<256, 28, 0x5555555u, 4, true, 2, false, false, 64>;  // window 2, look-back groups of 64
 using Cfg32_4 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 32>;  // look-back groups of 32
 using Cfg32_5 = OsCfg<256, 28, 0x5555555u, 4, true, 6, false, false, 32>;  // window 6, groups of 32
 using Cfg32_6 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, true>;       // count atomic's return = rank
-using Cfg32_7 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 8>;   // window 4, groups of 8
+using Cfg32_7 = OsCfg<256, 28, 0x5555555u, 4, true, 1, false, false, 32>;  // window 1, groups of 32
 using Cfg32_8 = OsCfg<256, 24, 0x555555u, 5, true, 2, false, false, 32>;   // 6144-key tiles, 5 blocks/SM (40 warps)
 using Cfg32_9 = OsCfg<256, 20, 0x55555u, 6, true, 2, false, false, 32>;    // 5120-key tiles, 6 blocks/SM (48 warps)
 using Cfg64_0 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 16>;     // prefetch, groups of 16 (best)
