@@ -366,7 +366,7 @@ def main():
         try:
             with open(prof) as f:
                 pj = json.load(f)
-            if pj.get("keys_per_launch"):
+            if pj.get("keys_per_launch") and pj.get("key_type", "u32") == kt:  # (the capture is of u32 keys)
                 traffic = pj["dram_bytes_per_launch"] * c / pj["keys_per_launch"]
         except Exception:
             traffic = None
