@@ -337,12 +337,14 @@ def test_small_sort_graph_replay(ms, kt):
         ctx.close()
 
 
-def test_msort_sort_host_pointer(ms):
-    n = 100003
-    a = mi.np_generate(n, "f32", "uniform", seed=9)
+@pytest.mark.parametrize("n,kt", [(100003, "f32"), ((1 << 21) + 1, "u32"), ((1 << 20) + 6, "u64")])
+def test_msort_sort_host_pointer(ms, n, kt):
+    """The north-star entry msort_sort on PAGEABLE host memory (numpy), below and above the pipelining
+    threshold (2^20 keys): the copies are staged by the driver, the result is the oracle's."""
+    a = mi.np_generate(n, kt, "uniform", seed=9)
     h = a.copy()
-    ms.msort_sort(h.ctypes.data, n, "f32", 1)
-    assert np.array_equal(h.view(np.uint32), sort.oracle_sort(a, "f32").view(np.uint32))
+    ms.msort_sort(h.ctypes.data, n, kt, 1)
+    assert bits(h, kt).tobytes() == bits(sort.oracle_sort(a, kt), kt).tobytes()
 
 
 def test_errors(ms):
