@@ -361,6 +361,7 @@ def main():
     alg_bytes = 2 * K * c
     achieved = alg_bytes / (pass_avg_ms / 1e3) / 1e9 if pass_avg_ms > 0 else None
     traffic = None
+    smem_pipe = None
     prof = os.path.join(ROOT, "profiles", "onesweep_traffic.json")
     if os.path.exists(prof):
         try:
@@ -368,12 +369,18 @@ def main():
                 pj = json.load(f)
             if pj.get("keys_per_launch") and pj.get("key_type", "u32") == kt:  # (the capture is of u32 keys)
                 traffic = pj["dram_bytes_per_launch"] * c / pj["keys_per_launch"]
+                if pj.get("smem_wavefronts_per_32_keys"):
+                    # the pass's binding resource (ncu, same capture): shared-memory wavefronts
+                    smem_pipe = {"wavefronts_per_32_keys": pj["smem_wavefronts_per_32_keys"],
+                                 "pct_of_peak": pj.get("smem_wavefronts_pct_of_peak_sustained_elapsed"),
+                                 "bank_conflicts_per_launch": pj.get("smem_bank_conflicts_per_launch"),
+                                 "source": "profiles/onesweep_traffic.json (ncu --set full capture)"}
         except Exception:
             traffic = None
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": (achieved / peak) if achieved else None, "traffic": traffic,
                 "kernel": "onesweep_kernel (S3 pass)", "alg_bytes_per_launch": alg_bytes,
-                "mean_launch_ms": pass_avg_ms, "peak_source": peak_src,
+                "mean_launch_ms": pass_avg_ms, "peak_source": peak_src, "smem_pipe": smem_pipe,
                 "whole_sort_hbm_frac": ((1 + 2 * (K * 8 // 8)) * K * c / (ms_per_step / 1e3) / 1e9 / peak) if g == 1 else None}
 
     # --- end to end through the public host API
