@@ -362,19 +362,20 @@ def main():
     achieved = alg_bytes / (pass_avg_ms / 1e3) / 1e9 if pass_avg_ms > 0 else None
     traffic = None
     smem_pipe = None
-    prof = os.path.join(ROOT, "profiles", "onesweep_traffic.json")
+    # one capture per key type: onesweep_traffic.json (u32), onesweep_traffic_<kt>.json (others)
+    prof = os.path.join(ROOT, "profiles", "onesweep_traffic.json" if kt == "u32" else f"onesweep_traffic_{kt}.json")
     if os.path.exists(prof):
         try:
             with open(prof) as f:
                 pj = json.load(f)
-            if pj.get("keys_per_launch") and pj.get("key_type", "u32") == kt:  # (the capture is of u32 keys)
+            if pj.get("keys_per_launch") and pj.get("key_type", "u32") == kt:  # (a capture of the same key type only)
                 traffic = pj["dram_bytes_per_launch"] * c / pj["keys_per_launch"]
                 if pj.get("smem_wavefronts_per_32_keys"):
                     # the pass's binding resource (ncu, same capture): shared-memory wavefronts
                     smem_pipe = {"wavefronts_per_32_keys": pj["smem_wavefronts_per_32_keys"],
                                  "pct_of_peak": pj.get("smem_wavefronts_pct_of_peak_sustained_elapsed"),
                                  "bank_conflicts_per_launch": pj.get("smem_bank_conflicts_per_launch"),
-                                 "source": "profiles/onesweep_traffic.json (ncu --set full capture)"}
+                                 "source": os.path.relpath(prof, ROOT) + " (ncu --set full capture)"}
         except Exception:
             traffic = None
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
