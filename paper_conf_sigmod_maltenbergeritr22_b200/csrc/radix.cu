@@ -187,8 +187,9 @@ __device__ __forceinline__ uint32_t ballot_match8(uint32_t d) {
 // THREADS x ITEMS keys per tile; bit i of BALLOT_MASK: item i ranks with the
 // ballot match (else smem atomicOr); MINB blocks per SM for __launch_bounds__.
 template <int THREADS_, int ITEMS_, uint32_t BALLOT_MASK_, int MINB_, bool PF_, int LB_ = 4, bool ELB_ = false,
-          bool CR_ = false, int GROUP_ = 8>
+          bool CR_ = false, int GROUP_ = 8, bool ECL_ = false>
 struct OsCfg {
+    static constexpr bool kEarlyClaim = ECL_;  // prefetch configs: claim the next tile before (not after) the look-back
     static constexpr uint32_t kGroup = GROUP_;  // look-back group size (tiles); 0 = tile-by-tile walk only
     static constexpr bool kCountRank = CR_;  // atomic-ranked passes: rank = the count atomic's return
     static constexpr bool kEarlyLookback = ELB_;  // look back right after publishing (before the ranking)
@@ -536,11 +537,14 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
         // --- look-back (deferred until after the ranking unless kEarlyLookback)
         if (tid < kRadix) {
             const int d = tid;
+            // kEarlyClaim: the claim's round trip overlaps thread 0's look-back
+            uint32_t claimed = 0;
+            if (Cfg::kPrefetch && Cfg::kEarlyClaim && tid == 0) claimed = atomicAdd(tile_counter, 1u);
             const uint32_t excl = Cfg::kEarlyLookback ? excl_early : lookback(d, tile, my_total);
             s_delta[d] = base[d] + excl - my_start;
             // Prefetch configs claim the next tile here so that its loads can
             // be issued before (and overlap) this tile's scatter.
-            if (Cfg::kPrefetch && tid == 0) s_next = atomicAdd(tile_counter, 1u);
+            if (Cfg::kPrefetch && tid == 0) s_next = Cfg::kEarlyClaim ? claimed : atomicAdd(tile_counter, 1u);
         }
         __syncthreads();
         if (!Cfg::kPrefetch && tid == 0) {
@@ -595,10 +599,12 @@ using Cfg32_6 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, true>;       // co
 using Cfg32_7 = OsCfg<256, 28, 0x5555555u, 4, true, 1, false, false, 32>;  // window 1, groups of 32
 using Cfg32_8 = OsCfg<256, 24, 0x555555u, 5, true, 2, false, false, 32>;   // 6144-key tiles, 5 blocks/SM (40 warps)
 using Cfg32_9 = OsCfg<256, 20, 0x55555u, 6, true, 2, false, false, 32>;    // 5120-key tiles, 6 blocks/SM (48 warps)
+using Cfg32_10 = OsCfg<256, 28, 0x5555555u, 4, true, 2, false, false, 32, true>;  // config 0 + next tile claimed before the look-back
 using Cfg64_0 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 16>;     // prefetch, groups of 16 (best)
 using Cfg64_1 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 0>;      // tile-by-tile look-back only
 using Cfg64_2 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 8>;      // groups of 8
 using Cfg64_3 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 32>;     // groups of 32
+using Cfg64_4 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 16, true>;  // config 0 + next tile claimed before the look-back
 
 constexpr uint32_t kMinTile32 = 256 * 20;  // smallest u32 tile above (sizes the status array)
 constexpr uint32_t kMinTile64 = 256 * 14;  // smallest u64 tile above
@@ -608,7 +614,7 @@ int env_cfg() {
     if (v < 0) {
         const char* e = std::getenv("MSORT_OS_CFG");
         v = e ? std::atoi(e) : 0;
-        if (v < 0 || v > 9) v = 0;
+        if (v < 0 || v > 10) v = 0;
     }
     return v;
 }
@@ -710,6 +716,7 @@ cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, c
             case 7: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_7, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
             case 8: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_8, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
             case 9: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_9, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 10: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_10, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
             default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
         }
     } else {
@@ -717,7 +724,8 @@ cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, c
             case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_1, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
             case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_2, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
             case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_3, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 4: case 5: case 6: case 7: case 8: case 9:
+            case 4: case 10: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_4, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 5: case 6: case 7: case 8: case 9:
                 return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
             default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
         }
@@ -776,12 +784,13 @@ static uint64_t active_group(int kt) {
     const int c = env_cfg();
     uint32_t gsz;
     if (key_bytes(kt) == 4) {
-        constexpr uint32_t G32[10] = {Cfg32_0::kGroup, Cfg32_1::kGroup, Cfg32_2::kGroup, Cfg32_3::kGroup, Cfg32_4::kGroup,
-                                      Cfg32_5::kGroup, Cfg32_6::kGroup, Cfg32_7::kGroup, Cfg32_8::kGroup, Cfg32_9::kGroup};
+        constexpr uint32_t G32[11] = {Cfg32_0::kGroup, Cfg32_1::kGroup, Cfg32_2::kGroup, Cfg32_3::kGroup, Cfg32_4::kGroup,
+                                      Cfg32_5::kGroup, Cfg32_6::kGroup, Cfg32_7::kGroup, Cfg32_8::kGroup, Cfg32_9::kGroup,
+                                      Cfg32_10::kGroup};
         gsz = G32[c];
     } else {
-        constexpr uint32_t G64[4] = {Cfg64_0::kGroup, Cfg64_1::kGroup, Cfg64_2::kGroup, Cfg64_3::kGroup};
-        gsz = G64[c < 4 ? c : 0];
+        constexpr uint32_t G64[5] = {Cfg64_0::kGroup, Cfg64_1::kGroup, Cfg64_2::kGroup, Cfg64_3::kGroup, Cfg64_4::kGroup};
+        gsz = G64[c == 10 ? 4 : (c < 5 ? c : 0)];
     }
     return gsz ? gsz : kMinGroup;
 }
