@@ -612,7 +612,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
 }
 // Tile configurations (selectable with MSORT_OS_CFG for tuning; 0 = default).
 // OsCfg<threads, keys/thread, ballot mask, blocks/SM, prefetch, look-back
-// window, look-back before ranking, count-rank, look-back group>; measured on
+// window, look-back before ranking, count-rank, look-back group, count at end>; measured on
 // B200 in profiles/radix_tuning_r1.md: config 0 is the fastest for both key
 // widths; the others stay selectable for tuning.
 using Cfg32_0 = OsCfg<256, 28, 0x5555555u, 4, true, 2, false, false, 32, true>;  // 7168-key tiles, 4 blocks of 256,
