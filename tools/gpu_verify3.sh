@@ -9,4 +9,7 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:onesweep -s 6 -c 1 -o gpurun_out/os_v3 python tools/prof_radix.py 4e9 u32 2 > /dev/null 2>&1
 timeout 600 python bench.py --key-type f32 --keys 2e9 --steps 5 --warmup 3 --het > gpurun_out/bench_c5_f32_v3.json 2>/dev/null
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:onesweep -s 2 -c 1 -o gpurun_out/os_f32_v3 python tools/prof_radix.py 2e9 f32 2 > /dev/null 2>&1
+python tools/ncu_summary.py gpurun_out/os_v3.ncu-rep 12 > gpurun_out/os_v3_summary.txt 2>&1
+python tools/ncu_summary.py gpurun_out/os_f32_v3.ncu-rep 12 > gpurun_out/os_f32_v3_summary.txt 2>&1
+rm -f gpurun_out/*.ncu-rep   # (gpurun brings back at most 64 MiB)
 echo done
