@@ -628,6 +628,8 @@ using Cfg32_7 = OsCfg<256, 28, 0x5555555u, 4, true, 1, false, false, 32>;  // wi
 using Cfg32_8 = OsCfg<256, 24, 0x555555u, 5, true, 2, false, false, 32>;   // 6144-key tiles, 5 blocks/SM (40 warps)
 using Cfg32_9 = OsCfg<256, 20, 0x55555u, 6, true, 2, false, false, 32>;    // 5120-key tiles, 6 blocks/SM (48 warps)
 using Cfg32_10 = OsCfg<256, 28, 0x5555555u, 4, true, 2, false, false, 32>;  // config 0 with the count at the tile's start (4 barriers)
+using Cfg32_11 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 32, true>;  // config 0 with look-back window 4
+using Cfg32_12 = OsCfg<256, 28, 0x5555555u, 4, true, 2, false, false, 16, true>;  // config 0 with look-back groups of 16
 using Cfg64_0 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 16>;     // prefetch, groups of 16 (best)
 using Cfg64_1 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 0>;      // tile-by-tile look-back only
 using Cfg64_2 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 8>;      // groups of 8
@@ -642,7 +644,7 @@ int env_cfg() {
     if (v < 0) {
         const char* e = std::getenv("MSORT_OS_CFG");
         v = e ? std::atoi(e) : 0;
-        if (v < 0 || v > 10) v = 0;
+        if (v < 0 || v > 12) v = 0;
     }
     return v;
 }
@@ -745,6 +747,8 @@ cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, c
             case 8: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_8, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
             case 9: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_9, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
             case 10: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_10, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 11: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_11, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+            case 12: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_12, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
             default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
         }
     } else {
@@ -812,13 +816,13 @@ static uint64_t active_group(int kt) {
     const int c = env_cfg();
     uint32_t gsz;
     if (key_bytes(kt) == 4) {
-        constexpr uint32_t G32[11] = {Cfg32_0::kGroup, Cfg32_1::kGroup, Cfg32_2::kGroup, Cfg32_3::kGroup, Cfg32_4::kGroup,
+        constexpr uint32_t G32[13] = {Cfg32_0::kGroup, Cfg32_1::kGroup, Cfg32_2::kGroup, Cfg32_3::kGroup, Cfg32_4::kGroup,
                                       Cfg32_5::kGroup, Cfg32_6::kGroup, Cfg32_7::kGroup, Cfg32_8::kGroup, Cfg32_9::kGroup,
-                                      Cfg32_10::kGroup};
+                                      Cfg32_10::kGroup, Cfg32_11::kGroup, Cfg32_12::kGroup};
         gsz = G32[c];
     } else {
         constexpr uint32_t G64[5] = {Cfg64_0::kGroup, Cfg64_1::kGroup, Cfg64_2::kGroup, Cfg64_3::kGroup, Cfg64_4::kGroup};
-        gsz = G64[c == 10 ? 4 : (c < 5 ? c : 0)];
+        gsz = G64[c == 10 ? 4 : (c < 5 ? c : 0)];  // (11, 12: u32 only)
     }
     return gsz ? gsz : kMinGroup;
 }
