@@ -1,8 +1,12 @@
-// HET sort baseline (comparison only, never the product path): the CPU side of
-// the paper's heterogeneous sort, §5.3: the g sorted GPU
-// chunks are merged on the host with a parallel multiway merge
-// (gnu_parallel::multiway_merge, a loser tree).  Keys compare by
-// the T order of DESIGN.md reading Q1 (floats: IEEE totalOrder on bits).
+// CPU baselines (comparison only, never the product path):
+//   het_multiway_merge  the CPU side of the paper's heterogeneous sort, PAPER.md
+//                       §5.3: the g sorted GPU chunks are merged on
+//                       the host with a parallel multiway merge
+//                       (gnu_parallel::multiway_merge, a loser tree)
+//   cpu_parallel_sort   GNU parallel mode's sort on all host cores - one of the
+//                       paper's CPU library baselines (§6 "CPU Sort Baseline",
+//                       P:2258-2266), reported beside the single-thread oracle
+// Keys compare by the T order of DESIGN.md reading Q1 (floats: IEEE totalOrder on bits).
 #include <parallel/algorithm>
 #include <omp.h>
 
@@ -48,6 +52,24 @@ extern "C" int het_multiway_merge(const void* const* runs, const uint64_t* lens,
         case 1: return merge<uint64_t, false>(runs, lens, k, out, threads);
         case 2: return merge<uint32_t, true>(runs, lens, k, out, threads);
         case 3: return merge<uint64_t, true>(runs, lens, k, out, threads);
+        default: return 1;
+    }
+}
+
+template <typename U, bool FLOAT>
+int psort(void* keys, uint64_t n, int threads) {
+    if (threads > 0) omp_set_num_threads(threads);
+    U* p = static_cast<U*>(keys);
+    __gnu_parallel::sort(p, p + n, TLess<U, FLOAT>(), __gnu_parallel::default_parallel_tag(threads > 0 ? threads : 0));
+    return 0;
+}
+
+extern "C" int cpu_parallel_sort(void* keys, uint64_t n, int key_type, int threads) {
+    switch (key_type) {
+        case 0: return psort<uint32_t, false>(keys, n, threads);
+        case 1: return psort<uint64_t, false>(keys, n, threads);
+        case 2: return psort<uint32_t, true>(keys, n, threads);
+        case 3: return psort<uint64_t, true>(keys, n, threads);
         default: return 1;
     }
 }

@@ -4,24 +4,33 @@
 Workload (BASELINE.json configs[2], paper Fig.1 shape): 4e9 uniform uint32 keys
 (16 GB), sorted on N = 1/2/4/8 GPUs (strong scaling: the total is fixed).  A
 "step" is one whole sort: per-GPU radix sort (S1-S3) and, for N > 1, the merge
-phase: by default NEXT-1, the paper's future work for NVSwitch systems
-(one all-to-all exchange fused into a local merge tree), with the
-paper's own g-1 merge stages (Alg.2, S4-S7) timed beside it as `alg2`
-(`--exchange 0` makes Alg.2 the measured path).
+phase - the paper's g-1 merge stages (Alg.2, S4-S7) with the
+exchange fused into the merge and every stage decided on the GPUs; NEXT-1, the
+paper's future work for NVSwitch systems (one all-to-all exchange),
+is timed beside it as `next1` with equal standing (`--exchange 2` makes it the
+headline).
 
   value  device-resident keys/s: chunks already in HBM; CUDA events on the
          stream the sort is ordered on, max over ranks; the input is restored
          from a pristine copy between steps OUTSIDE the event pair (inputs are
-         16 GB >> 126 MB L2, so no L2 flush is needed)
+         16 GB >> 126 MB L2, so no L2 flush is needed); the output of the last
+         step is verified (sorted + multiset fingerprint) -> `verified`
   e2e    the same metric through the public host-pointer API (msort_sort_host /
          msort_dist_sort_host): pinned host keys -> H2D -> sort -> D2H, timed
          per call; N = 1: the pipelined path (transfers overlapped with the
-         sort), the sequential one interleaved with it as `e2e.sequential`
+         sort), the sequential one interleaved with it as `e2e.sequential`;
+         `e2e.pcie` = the achieved H2D / D2H rates against the in-run measured
+         parallel PCIe peaks (msort_measure_links, P:664-709 pattern)
   roofline  dominant kernel = the onesweep pass (S3): algorithmic bytes
          2*K*c per launch / mean launch time (library CUDA events around each
          launch) vs MEASURED_PEAKS.json hbm_gbs
+  nvlink N > 1: per Alg.2 stage the busiest mirrored pair's bytes (x_d * K) /
+         the stage's exchange time (max over ranks) against 900 GB/s per
+         direction and against the in-run measured mirrored-pair peak
+         (msort_measure_links: GPU i <-> GPU g-1-i concurrently)
   cpu_baseline  the oracle (np.sort on T codes, single thread) on a bounded
-         sample of the same workload, on this host
+         sample of the same workload, on this host; `.parallel` = GNU parallel
+         mode's sort on all host cores on a >= 2^28-key sample
 
 `--impl reference` times the oracle itself (the reference arm of this tier).
 """
@@ -30,6 +39,7 @@ from __future__ import annotations
 import argparse
 import json
 import os
+import platform
 import subprocess
 import sys
 import threading
@@ -41,6 +51,9 @@ sys.path.insert(0, ROOT)
 N_DEFAULT = 4_000_000_000
 PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FALLBACK_HBM = 6650.0
+NVLINK_NOMINAL_GBS = 900.0  # NVLink 5 per direction per GPU (north_star)
+EXCHANGE_NAMES = ["Alg.2, fused peer-read merge, stages decided on the GPUs", "Alg.2, swap then merge",
+                  "NEXT-1 single all-to-all fused into the merge", "NEXT-1 single all-to-all, pull then merge"]
 PAPER_CONTEXT = {
     "source": "PAPER.md P:124-141 (Fig.1), DGX A100, 16 GB = 4e9 ints, end-to-end",
     "thrust_1gpu_s": 1.47, "p2p_2gpu_s": 0.75, "p2p_4gpu_s": 0.45, "het_2gpu_s": 1.09, "het_4gpu_s": 0.75,
@@ -48,7 +61,7 @@ PAPER_CONTEXT = {
 }
 
 
-def parse():
+def parse(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
@@ -60,17 +73,19 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-links", action="store_true", help="skip the interconnect peak measurement")
     ap.add_argument("--seed", type=int, default=1)
-    ap.add_argument("--exchange", type=int, default=None,
-                    help="merge phase for N>1: 0 the paper's Alg.2 with fused exchange+merge, 1 Alg.2 swap then "
-                         "merge (single process only), 2 (default for N>1) NEXT-1 - the paper's future work for "
-                         "NVSwitch systems, P:3416-3424 - single all-to-all fused into the merge, 3 NEXT-1 pull then "
-                         "merge. With 2 or 3, Alg.2 (0) is timed too and reported as `alg2`")
-    ap.add_argument("--no-alg2", action="store_true", help="N>1: skip the Alg.2 comparison timing")
-    ap.add_argument("--het", action="store_true", help="also time the HET-sort baseline (GPU chunk sort + CPU merge)")
+    ap.add_argument("--exchange", type=int, default=0,
+                    help="merge phase for N>1: 0 (default) the paper's Alg.2, fused exchange+merge, decided on the "
+                         "GPUs; 2 NEXT-1 (P:3416-3424) single all-to-all fused into the merge; 3 NEXT-1 pull then "
+                         "merge. The other of {0, 2} is timed too and reported beside it")
+    ap.add_argument("--no-compare", action="store_true", help="N>1: skip the second merge-phase variant")
+    ap.add_argument("--het", action="store_true", help="also time the HET-sort baseline (GPU chunk sorts + CPU merge)")
     ap.add_argument("--het-chunks", type=int, default=8)
+    ap.add_argument("--het-gpus", type=int, default=0, help="GPUs for the HET chunk sorts (0: all visible)")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
-    return ap.parse_args()
+    ap.add_argument("--cpu-parallel-keys", type=float, default=float(1 << 28))
+    return ap.parse_args(argv)
 
 
 def hbm_peak():
@@ -169,10 +184,19 @@ class ClockSampler:
                 "samples": len(self.rows), "source": "nvml" if self.nv is not None else "nvidia-smi"}
 
 
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return platform.processor() or "unknown"
+
+
 def cpu_baseline(n_total: int, key_type: str, dist: str, seed: int, seconds: float):
     """The oracle as it stands (np.sort on T codes, one thread) on a bounded sample."""
-    import numpy as np
-
     import msort_inputs as mi
     from oracle import sort as osort
     sample = min(n_total, 1 << 26)
@@ -184,9 +208,32 @@ def cpu_baseline(n_total: int, key_type: str, dist: str, seed: int, seconds: flo
         el = time.perf_counter() - t0
         if el >= seconds:
             break
-    return {"value": done / el, "unit": "keys/s", "cores": 1, "kind": "oracle",
+    return {"value": done / el, "unit": "keys/s", "cores": 1, "kind": "oracle", "cpu_model": cpu_model(),
             "sample": f"first {sample} keys of the {n_total}-key {dist} {key_type} workload, "
                       f"oracle.sort.oracle_sort (np.sort of T codes) repeated {done // sample}x in {el:.1f} s"}
+
+
+def cpu_parallel_baseline(pristine, n_total: int, key_type: str, count: int):
+    """GNU parallel mode's sort (__gnu_parallel::sort, all host cores) on the first `count` keys of the
+    workload (copied from the GPU-generated input); the paper's CPU library baseline family."""
+    import torch
+
+    from baseline import het
+    count = int(min(count, pristine.numel()))
+    host = torch.empty(count, dtype=pristine.dtype, pin_memory=True)
+    src = pristine[:count].cpu()
+    kt = {"u32": 0, "u64": 1, "f32": 2, "f64": 3}[key_type]
+    times = []
+    for _ in range(2):
+        host.copy_(src)
+        t0 = time.perf_counter()
+        het.cpu_parallel_sort(host.data_ptr(), count, kt, 0)
+        times.append(time.perf_counter() - t0)
+    el = min(times)
+    threads = het.max_threads()
+    return {"value": count / el, "unit": "keys/s", "cores": threads, "kind": "__gnu_parallel::sort",
+            "cpu_model": cpu_model(), "seconds": el,
+            "sample": f"first {count} keys of the {n_total}-key workload, best of 2, {threads} OpenMP threads"}
 
 
 def run_reference(args):
@@ -194,8 +241,6 @@ def run_reference(args):
     if rank != 0:
         return
     cb = cpu_baseline(args.n, args.key_type, args.dist, args.seed, max(1.0, args.cpu_seconds / 2))
-    import numpy as np
-
     import msort_inputs as mi
     from oracle import sort as osort
     sample = min(args.n, 1 << 25)
@@ -219,13 +264,105 @@ def run_reference(args):
     }))
 
 
+# --- output verification (torch on the GPU; a check of the timed result, not the product path) -------------
+
+_MIX1, _MIX2 = -0x2917014799A6026D, -0x40A7B892E31B1A47  # 0xD6E8FEB86659FD93, 0xBF58476D1CE4E5B9 as int64
+
+
+def _order_codes(x, kt):
+    """int64 values whose signed order is the T order of the keys (reading Q1)."""
+    import torch
+    if kt in ("u32", "f32"):
+        u = x.view(torch.int32).to(torch.int64) & 0xFFFFFFFF
+        if kt == "f32":
+            u = torch.where(u >= (1 << 31), u ^ 0xFFFFFFFF, u | (1 << 31))
+        return u
+    u = x.view(torch.int64)
+    if kt == "f64":  # negatives: all bits flipped; then the unsigned order = signed order after a sign flip
+        return torch.where(u < 0, ~u ^ (-(1 << 63)), u)
+    return u ^ (-(1 << 63))
+
+
+def _fingerprint(codes):
+    import torch
+    h1 = codes * _MIX1
+    h1 = h1 ^ ((h1 >> 29) & ((1 << 35) - 1))
+    h2 = (codes + 0x1234567) * _MIX2
+    h2 = h2 ^ ((h2 >> 31) & ((1 << 33) - 1))
+    return int(h1.sum().item()) % (1 << 64), int(h2.sum().item()) % (1 << 64), int(codes.numel())
+
+
+def verify_local(out, inp, valid, kt, block=1 << 27):
+    """This rank: out[:valid] non-decreasing under T, and the multiset fingerprint of out[:valid] and
+    inp[:valid]; first / last codes for the cross-rank boundary check."""
+    ok, last, first = True, None, None
+    fo, fi = [0, 0, 0], [0, 0, 0]
+    for off in range(0, valid, block):
+        hi = min(valid, off + block)
+        c = _order_codes(out[off:hi], kt)
+        ok = ok and bool((c[1:] >= c[:-1]).all().item()) and (last is None or last <= int(c[0].item()))
+        first = int(c[0].item()) if first is None else first
+        last = int(c[-1].item())
+        a = _fingerprint(c)
+        b = _fingerprint(_order_codes(inp[off:hi], kt))
+        fo = [(fo[0] + a[0]) % (1 << 64), (fo[1] + a[1]) % (1 << 64), fo[2] + a[2]]
+        fi = [(fi[0] + b[0]) % (1 << 64), (fi[1] + b[1]) % (1 << 64), fi[2] + b[2]]
+    return {"sorted": ok, "first": first, "last": last, "fp_out": fo, "fp_in": fi}
+
+
+def verify_all(local, dist):
+    """Combine the ranks' verify_local results (rank order)."""
+    parts = [local]
+    if dist is not None:
+        parts = [None] * dist.get_world_size()
+        dist.all_gather_object(parts, local)
+    ok = all(p["sorted"] for p in parts)
+    prev = None
+    for p in parts:
+        if p["first"] is None:
+            continue
+        ok = ok and (prev is None or prev <= p["first"])
+        prev = p["last"]
+
+    def tot(k):
+        return [sum(p[k][0] for p in parts) % (1 << 64), sum(p[k][1] for p in parts) % (1 << 64),
+                sum(p[k][2] for p in parts)]
+    ok = ok and tot("fp_out") == tot("fp_in")
+    return {"verified": bool(ok), "method": "every rank's output non-decreasing under T, rank boundaries ordered, "
+                                            "and out/in multiset fingerprints (2 x sum of mixed codes) equal"}
+
+
+# --- interconnect fractions ---------------------------------------------------------------------------------
+
+def nvlink_fractions(stages: dict, K: int, peaks: dict | None, same_device: bool):
+    """Per merge stage: busiest mirrored pair's bytes / the stage's exchange time."""
+    rows = []
+    for s, (lab, mx, ms) in enumerate(zip(stages["stage_label"], stages["stage_max_x"], stages["stage_exchange_ms"])):
+        b = mx * K
+        gbs = b / (ms * 1e6) if ms > 0 else None
+        row = {"stage": s, "label": lab, "busiest_pair_bytes": b, "exchange_ms": ms, "achieved_gbs": gbs,
+               "frac_of_900": (gbs / NVLINK_NOMINAL_GBS) if gbs else None}
+        if peaks and peaks.get("p2p_ce_gbs"):
+            row["frac_of_measured_ce"] = gbs / peaks["p2p_ce_gbs"] if gbs else None
+            row["frac_of_measured_sm"] = gbs / peaks["p2p_sm_gbs"] if gbs and peaks.get("p2p_sm_gbs") else None
+        rows.append(row)
+    tot_b = sum(r["busiest_pair_bytes"] for r in rows)
+    tot_ms = sum(r["exchange_ms"] for r in rows)
+    agg = tot_b / (tot_ms * 1e6) if tot_ms > 0 else None
+    return {"per_stage": rows, "busiest_pair_bytes_total": tot_b, "exchange_ms_total": tot_ms, "achieved_gbs": agg,
+            "frac_of_900": (agg / NVLINK_NOMINAL_GBS) if agg else None,
+            "frac_of_measured_ce": (agg / peaks["p2p_ce_gbs"]) if agg and peaks and peaks.get("p2p_ce_gbs") else None,
+            "nominal_gbs": NVLINK_NOMINAL_GBS, "measured_peaks": peaks,
+            "note": ("ranks share one GPU: the 'pairs' are HBM copies, not NVLink" if same_device else
+                     "distinct GPUs: NVLink 5 through NVSwitch")}
+
+
 def main():
     args = parse()
     args.n = int(args.n)
     if args.impl == "reference":
         run_reference(args)
         return
-    import numpy as np
     import torch
 
     import msort_inputs as mi
@@ -234,12 +371,12 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world != args.gpus:
-        if world == 1 and args.gpus > 1:
-            raise SystemExit("--gpus N > 1 runs under torchrun (one process per GPU)")
+    if world != args.gpus and world == 1 and args.gpus > 1:
+        raise SystemExit("--gpus N > 1 runs under torchrun (one process per GPU)")
     # MSORT_BENCH_SAME_GPU=1 maps every rank to cuda:0 (testing the N>1 path on a
     # one-GPU box: CUDA IPC works between processes on one device)
-    if os.environ.get("MSORT_BENCH_SAME_GPU") == "1":
+    same_gpu = os.environ.get("MSORT_BENCH_SAME_GPU") == "1"
+    if same_gpu:
         local = 0
     torch.cuda.set_device(local)
     dist = None
@@ -252,30 +389,26 @@ def main():
     kt = args.key_type
     K = mi.KEY_BYTES[kt]
     n = args.n
-    c = ((n + g - 1) // g + 3) // 4 * 4
-    n_valid_local = max(0, min(n - rank * c, c))
+    if g == 1:
+        c, off, valid = n, 0, n
+    else:
+        c, off, valid = ms.msort_plan_chunk(n, g, rank)   # the library's chunking rule (reading Q3)
     dev = torch.device("cuda", local)
     tdt = mi.torch_dtype(kt)
 
-    # --- input: this rank's chunk of the global seeded workload, generated on the GPU
+    # --- input: this rank's slice of the global seeded workload, generated on the GPU (the library pads)
     pristine = torch.empty(c, dtype=tdt, device=dev)
-    mi.t_generate_into(pristine[:n_valid_local], n, kt, args.dist, seed=args.seed, start=rank * c, block=1 << 27)
-    if n_valid_local < c:
-        # reading Q3 padding: largest key under T
-        pad = {"u32": -1, "u64": -1, "f32": 0x7FFFFFFF, "f64": 0x7FFFFFFFFFFFFFFF}[kt]
-        pristine.view(torch.int32 if K == 4 else torch.int64)[n_valid_local:] = pad
+    mi.t_generate_into(pristine[:valid], n, kt, args.dist, seed=args.seed, start=off, block=1 << 27)
     work = torch.empty_like(pristine)
     stream = torch.cuda.Stream(device=dev)
 
     if g == 1:
         ctx = ms.Context(1, c, kt, device_ids=[local])
-        sort_dev = lambda: ctx.sort_device([ms.tensor_ptr(work)], c, streams=[stream])  # noqa: E731
+        sort_dev = lambda: ctx.sort_device([ms.tensor_ptr(work)], n, streams=[stream])  # noqa: E731
     else:
         from paper_conf_sigmod_maltenbergeritr22_b200 import dist as mdist
         ctx = mdist.dist_context(rank, g, local, c, kt)
-        sort_dev = lambda: ctx.sort(ms.tensor_ptr(work), c, stream=stream)  # noqa: E731
-    if args.exchange is None:
-        args.exchange = 2 if g > 1 else 0
+        sort_dev = lambda: ctx.sort(ms.tensor_ptr(work), n, stream=stream)  # noqa: E731
     if g > 1:
         if args.exchange == 1:
             raise SystemExit("--exchange 1 (swap then merge) is a single-process option")
@@ -286,15 +419,41 @@ def main():
         if dist:
             dist.barrier()
 
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    def max_over_ranks(x: float) -> float:
+        if not dist:
+            return x
+        tt = torch.tensor([x], dtype=torch.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        return float(tt.item())
+
+    def timed_steps(steps):
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+        acc = {"pass_ms": 0.0, "pass_cnt": 0, "hist_ms": 0.0, "launches": 0, "tm": None, "stage_x_ms": None}
+        for i in range(steps):
+            with torch.cuda.stream(stream):
+                work.copy_(pristine)      # restore input: outside the event pair
+                ev[i][0].record(stream)
+            sort_dev()
+            with torch.cuda.stream(stream):
+                ev[i][1].record(stream)
+            tm = ctx.timings()
+            acc["pass_ms"] += tm["pass_ms_sum"]
+            acc["pass_cnt"] += tm["passes_run"]
+            acc["hist_ms"] += tm["hist_ms"]
+            acc["launches"] += tm["kernel_launches"]
+            acc["tm"] = tm
+        barrier()
+        step_ms = [a.elapsed_time(b) for a, b in ev]
+        acc["step_ms"] = step_ms
+        acc["ms_per_step"] = max_over_ranks(sum(step_ms)) / steps
+        return acc
+
     # warm-up (untimed)
     for _ in range(args.warmup):
         with torch.cuda.stream(stream):
             work.copy_(pristine)
         sort_dev()
     barrier()
-    pass_ms, pass_cnt, stage_info, launches = 0.0, 0, None, 0
-    hist_ms = 0.0
     try:
         pp = torch.cuda.get_device_properties(dev)
         pci = f"{pp.pci_domain_id:08X}:{pp.pci_bus_id:02X}:{pp.pci_device_id:02X}.0"
@@ -303,61 +462,50 @@ def main():
     with ClockSampler(local, pci) as clk:
         barrier()
         t_wall = time.perf_counter()
-        for i in range(args.steps):
-            with torch.cuda.stream(stream):
-                work.copy_(pristine)      # restore input: outside the event pair
-                ev[i][0].record(stream)
-            sort_dev()
-            with torch.cuda.stream(stream):
-                ev[i][1].record(stream)
-            tm = ctx.timings()
-            pass_ms += tm["pass_ms_sum"]
-            pass_cnt += tm["passes_run"]
-            hist_ms += tm["hist_ms"]
-            stage_info = tm
-            launches += tm["kernel_launches"]
-        barrier()
+        main_run = timed_steps(args.steps)
         wall = time.perf_counter() - t_wall
-    step_ms = [a.elapsed_time(b) for a, b in ev]
-    tot = sum(step_ms)
-    if dist:
-        tt = torch.tensor([tot], dtype=torch.float64)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        tot = float(tt.item())
-    ms_per_step = tot / args.steps
+    ms_per_step = main_run["ms_per_step"]
     value = n / (ms_per_step / 1e3)
+    stage_info = main_run["tm"]
+    verify = verify_all(verify_local(work, pristine, valid, kt), dist)
 
-    # --- N>1 with NEXT-1: the paper's own merge phase (Alg.2) timed the same way, as context
-    alg2 = None
-    if g > 1 and args.exchange in (2, 3) and not args.no_alg2:
-        ctx.set_option(ms.MSORT_OPT_EXCHANGE, 0)
+    # --- N>1: the other merge phase (NEXT-1 beside Alg.2, or Alg.2 beside NEXT-1), timed the same way
+    compare = None
+    if g > 1 and not args.no_compare:
+        other = 2 if args.exchange == 0 else 0
+        ctx.set_option(ms.MSORT_OPT_EXCHANGE, other)
         for _ in range(2):
             with torch.cuda.stream(stream):
                 work.copy_(pristine)
             sort_dev()
         barrier()
-        ev2 = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-        for i in range(args.steps):
-            with torch.cuda.stream(stream):
-                work.copy_(pristine)
-                ev2[i][0].record(stream)
-            sort_dev()
-            with torch.cuda.stream(stream):
-                ev2[i][1].record(stream)
-        barrier()
-        t2 = sum(a.elapsed_time(b) for a, b in ev2)
-        tt = torch.tensor([t2], dtype=torch.float64)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        ms2 = float(tt.item()) / args.steps
-        at = ctx.timings()
-        alg2 = {"value": n / (ms2 / 1e3), "unit": "keys/s", "ms_per_step": ms2,
-                "exchange": "Alg.2 (paper P:1763-1854), fused peer-read merge", "merge_phase_ms": at["merge_ms"],
-                "stage_label": at["stage_label"], "stage_max_x": at["stage_max_x"]}
+        r2 = timed_steps(args.steps)
+        v2 = verify_all(verify_local(work, pristine, valid, kt), dist)
+        at = r2["tm"]
+        compare = {"value": n / (r2["ms_per_step"] / 1e3), "unit": "keys/s", "ms_per_step": r2["ms_per_step"],
+                   "exchange": EXCHANGE_NAMES[other], "merge_phase_ms": max_over_ranks(at["merge_ms"]),
+                   "stage_label": at["stage_label"], "stage_max_x": at["stage_max_x"],
+                   "verified": v2["verified"]}
         ctx.set_option(ms.MSORT_OPT_EXCHANGE, args.exchange)
+
+    # --- interconnect peaks (msort_measure_links; every rank, collective in dist mode)
+    peaks = None
+    if not args.no_links:
+        try:
+            pk = ctx.measure_links(min(c * K, 4 << 30), 3)
+            if dist:  # the slowest rank's rates
+                for k in ("p2p_ce_gbs", "p2p_sm_gbs", "h2d_gbs", "d2h_gbs", "bidir_gbs"):
+                    tt = torch.tensor([pk[k]], dtype=torch.float64)
+                    dist.all_reduce(tt, op=dist.ReduceOp.MIN)
+                    pk[k] = float(tt.item())
+            pk["same_device"] = bool(same_gpu or pk.get("same_device") == 1)
+            peaks = pk
+        except ms.MsortError as e:
+            peaks = {"error": str(e)}
 
     # --- roofline of the dominant kernel (onesweep pass)
     peak, peak_src = hbm_peak()
-    pass_avg_ms = pass_ms / max(1, pass_cnt)
+    pass_avg_ms = main_run["pass_ms"] / max(1, main_run["pass_cnt"])
     alg_bytes = 2 * K * c
     achieved = alg_bytes / (pass_avg_ms / 1e3) / 1e9 if pass_avg_ms > 0 else None
     traffic = None
@@ -371,24 +519,34 @@ def main():
             if pj.get("keys_per_launch") and pj.get("key_type", "u32") == kt:  # (a capture of the same key type only)
                 traffic = pj["dram_bytes_per_launch"] * c / pj["keys_per_launch"]
                 if pj.get("smem_wavefronts_per_32_keys"):
-                    # the pass's binding resource (ncu, same capture): shared-memory wavefronts
                     smem_pipe = {"wavefronts_per_32_keys": pj["smem_wavefronts_per_32_keys"],
                                  "pct_of_peak": pj.get("smem_wavefronts_pct_of_peak_sustained_elapsed"),
                                  "bank_conflicts_per_launch": pj.get("smem_bank_conflicts_per_launch"),
                                  "source": os.path.relpath(prof, ROOT) + " (ncu --set full capture)"}
         except Exception:
             traffic = None
+    P = K  # passes (8-bit digits)
+    radix_bytes = (1 + 2 * P) * K * c
+    merging_stages = sum(1 for x in (stage_info["stage_max_x"] if g > 1 else []) if x) if g > 1 else 0
+    roof_ms = (radix_bytes + merging_stages * 2 * K * c) / (peak * 1e9) * 1e3
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": (achieved / peak) if achieved else None, "traffic": traffic,
                 "kernel": "onesweep_kernel (S3 pass)", "alg_bytes_per_launch": alg_bytes,
                 "mean_launch_ms": pass_avg_ms, "peak_source": peak_src, "smem_pipe": smem_pipe,
-                "whole_sort_hbm_frac": ((1 + 2 * (K * 8 // 8)) * K * c / (ms_per_step / 1e3) / 1e9 / peak) if g == 1 else None}
+                "whole_sort_hbm_frac": roof_ms / ms_per_step,
+                "whole_sort_model": "(radix (1+2P)K + 2K per merging stage) bytes per GPU / HBM peak / measured step"}
+
+    nvlink = None
+    if g > 1:
+        st = {k: stage_info[k] for k in ("stage_label", "stage_max_x")}
+        st["stage_exchange_ms"] = [max_over_ranks(x) for x in stage_info["stage_exchange_ms"]]
+        nvlink = nvlink_fractions(st, K, peaks if peaks and "error" not in peaks else None, same_gpu)
 
     # --- end to end through the public host API
     e2e = None
     if not args.no_e2e and args.e2e_steps > 0:
-        host = torch.empty(c if g > 1 else n, dtype=tdt, pin_memory=True)
-        host_pristine = pristine[: (c if g > 1 else n)].cpu()
+        host = torch.empty(valid, dtype=tdt, pin_memory=True)
+        host_pristine = pristine[:valid].cpu()
         # one GPU: the pipelined host path (MSORT_OPT_HOST_PIPELINE, the default)
         # is the e2e number; the sequential path (H2D, sort, D2H one after the
         # other) runs interleaved with it in the same process as context (PCIe
@@ -403,24 +561,31 @@ def main():
                 host.copy_(host_pristine)
                 barrier()
                 t0 = time.perf_counter()
-                if g == 1:
-                    ctx.sort_host(ms.tensor_ptr(host), n)
-                else:
-                    ctx.sort_host(ms.tensor_ptr(host), c)
-                el = time.perf_counter() - t0
-                if dist:
-                    tt = torch.tensor([el], dtype=torch.float64)
-                    dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-                    el = float(tt.item())
+                ctx.sort_host(ms.tensor_ptr(host), n)
+                el = max_over_ranks(time.perf_counter() - t0)
                 if i > 0:
                     times[v].append(el)
                     et = ctx.timings()
-                    phases[v] = {"h2d": et["h2d_ms"], "sort": et["sort_ms"], "merge": et["merge_ms"], "d2h": et["d2h_ms"]}
-        main = variants[0]
-        tm = sum(times[main]) / len(times[main])
+                    phases[v] = {"h2d": max_over_ranks(et["h2d_ms"]), "sort": max_over_ranks(et["sort_ms"]),
+                                 "merge": max_over_ranks(et["merge_ms"]), "d2h": max_over_ranks(et["d2h_ms"])}
+        main_v = variants[0]
+        tm = sum(times[main_v]) / len(times[main_v])
+        ph = phases[main_v]
         e2e = {"value": n / tm, "unit": "keys/s", "h2d_bytes_per_step": n * K,
-               "d2h_bytes_per_step": n * K, "ms_per_step": 1e3 * tm, "phases_ms": phases[main],
-               "steps": len(times[main])}
+               "d2h_bytes_per_step": n * K, "ms_per_step": 1e3 * tm, "phases_ms": ph,
+               "steps": len(times[main_v])}
+        # PCIe: this rank's bytes over its H2D / D2H phase vs the measured parallel peaks
+        pcie = {"h2d_gbs": valid * K / (ph["h2d"] * 1e6) if ph["h2d"] > 0 else None,
+                "d2h_gbs": valid * K / (ph["d2h"] * 1e6) if ph["d2h"] > 0 else None,
+                "serial_bound_ms": None}
+        if peaks and "error" not in peaks:
+            pcie["peak_h2d_gbs"], pcie["peak_d2h_gbs"] = peaks["h2d_gbs"], peaks["d2h_gbs"]
+            pcie["frac_h2d"] = pcie["h2d_gbs"] / peaks["h2d_gbs"] if pcie["h2d_gbs"] else None
+            pcie["frac_d2h"] = pcie["d2h_gbs"] / peaks["d2h_gbs"] if pcie["d2h_gbs"] else None
+            # the e2e time can't beat moving the bytes in and then out at the measured rates
+            pcie["serial_bound_ms"] = valid * K / (peaks["h2d_gbs"] * 1e6) + valid * K / (peaks["d2h_gbs"] * 1e6)
+            pcie["e2e_frac_of_serial_bound"] = pcie["serial_bound_ms"] / (1e3 * tm)
+        e2e["pcie"] = pcie
         if g == 1:
             e2e["path"] = "pipelined (4 H2D pieces sorted as they land, sliced final merge overlapped with D2H)"
             ts = sum(times[0]) / len(times[0])
@@ -430,20 +595,29 @@ def main():
     cpu = None
     if rank == 0 and g == 1 and not args.no_cpu:
         cpu = cpu_baseline(n, kt, args.dist, args.seed, args.cpu_seconds)
+        try:
+            cpu["parallel"] = cpu_parallel_baseline(pristine[:valid], n, kt, int(args.cpu_parallel_keys))
+        except Exception as e:  # (the HET/CPU helper library could not be built here)
+            cpu["parallel"] = {"error": str(e)}
 
     het = None
     if args.het and g == 1:
         from baseline import het as hetmod
-        hk = pristine[:n].cpu().pin_memory()
-        hetmod.het_sort_host(hk, kt, chunks=args.het_chunks)           # warm-up (allocations, OpenMP start)
-        hk.copy_(pristine[:n].cpu())
-        info = hetmod.het_sort_host(hk, kt, chunks=args.het_chunks)
+        ngpu = torch.cuda.device_count() if args.het_gpus <= 0 else min(args.het_gpus, torch.cuda.device_count())
+        hs = hetmod.HetSort(n, kt, chunks=args.het_chunks, devices=list(range(ngpu)))
+        hk = torch.empty(n, dtype=tdt, pin_memory=True)
+        src = pristine[:n].cpu()
+        hk.copy_(src)
+        hs.run(hk)                                    # warm-up (OpenMP start)
+        hk.copy_(src)
+        info = hs.run(hk)
         het = {"value": n / info["total_s"], "unit": "keys/s", "kind": "HET sort (paper §5.3): libmsort radix per "
-               f"chunk on 1 GPU + D2H + CPU multiway merge (libstdc++ parallel, {info['threads']} threads)",
-               "chunks": info["chunks"], "gpu_sort_and_copies_s": info["gpu_sort_and_copies_s"],
-               "cpu_merge_s": info["cpu_merge_s"]}
-        del hk
+               f"chunk on {info['gpus']} GPU(s) + D2H + CPU multiway merge (libstdc++ parallel, "
+               f"{info['threads']} threads); buffers pre-allocated", "chunks": info["chunks"], "gpus": info["gpus"],
+               "gpu_sort_and_copies_s": info["gpu_sort_and_copies_s"], "cpu_merge_s": info["cpu_merge_s"]}
+        del hk, src, hs
 
+    merge_phase_ms = max_over_ranks(stage_info["merge_ms"]) if stage_info else None
     if rank == 0:
         out = {
             "metric": "keys/sec", "value": value, "unit": "keys/s", "n_gpus": g, "steps": args.steps,
@@ -453,23 +627,28 @@ def main():
                                    f"device-resident P2P sort on {g} GPU(s)",
                        "n": n, "keys_per_gpu": c, "key_type": kt, "distribution": args.dist, "seed": args.seed,
                        "parallelism": f"p2p{g}", "l2": "inputs 16 GB >> 126 MB L2 (no flush needed)",
-                       "exchange": ["Alg.2, fused peer-read merge", "Alg.2, swap then merge",
-                                    "NEXT-1 single all-to-all fused into the merge", "NEXT-1 single all-to-all, pull then merge"][args.exchange] if g > 1 else "none (1 GPU)"},
-            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
+                       "exchange": EXCHANGE_NAMES[args.exchange] if g > 1 else "none (1 GPU)",
+                       "ranks_share_one_gpu": same_gpu},
+            "verified": verify["verified"], "verify_method": verify["method"],
+            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": main_run["launches"],
             "clocks": clk.summary(), "wall_s_timed_region": wall,
-            "step_ms": {"min": min(step_ms), "max": max(step_ms)},
-            "phases_ms": {"hist": hist_ms / args.steps, "onesweep_passes": pass_ms / args.steps,
-                          "merge_phase": stage_info["merge_ms"] if stage_info else None},
+            "step_ms": {"min": min(main_run["step_ms"]), "max": max(main_run["step_ms"])},
+            "phases_ms": {"hist": main_run["hist_ms"] / args.steps,
+                          "onesweep_passes": main_run["pass_ms"] / args.steps,
+                          "merge_phase": merge_phase_ms},
             "stages": {k: stage_info[k] for k in ("stage_label", "stage_pivot", "stage_max_x", "stage_ms",
                                                   "stage_exchange_ms")} if stage_info and g > 1 else None,
+            "nvlink": nvlink, "links": peaks,
             "paper_context": PAPER_CONTEXT,
             "het_baseline": het,
-            "alg2": alg2,
+            ("next1" if args.exchange == 0 else "alg2"): compare,
         }
         print(json.dumps(out))
     if dist:
         dist.barrier()
         dist.destroy_process_group()
+    if not verify["verified"]:
+        sys.exit(3)
 
 
 if __name__ == "__main__":

@@ -63,7 +63,7 @@ typedef enum {
     MSORT_ERR_DEVICE = 2,           /* too few GPUs, no peer access, no CUDA device                        */
     MSORT_ERR_OUT_OF_MEMORY = 3,    /* device or pinned allocation failed (no CPU fallback)                */
     MSORT_ERR_CUDA = 4,             /* a CUDA runtime call or kernel failed                                */
-    MSORT_ERR_NCCL = 5,             /* reserved                                                            */
+    MSORT_ERR_NCCL = 5,             /* libnccl missing, or an NCCL call failed (exchange mode 4)            */
     MSORT_ERR_INTERNAL = 6,         /* invariant violated inside the library                               */
     MSORT_ERR_TIMEOUT = 7           /* a cross-GPU device barrier did not complete (dist mode)             */
 } msort_status;
@@ -115,7 +115,15 @@ enum {
                                        a log2(g)-round merge tree whose first round reads the g runs straight
                                        from the peers' chunks over NVLink;
                                        3: NEXT-1 with the exchange as separate pulls (every GPU copies its run
-                                       from every chunk into a local buffer), then the merge tree            */
+                                       from every chunk into a local buffer), then the merge tree;
+                                       4: the swap as grouped ncclSend/ncclRecv per mirrored pair into a
+                                       receive buffer, then a local merge (north_star S5).  Single process:
+                                       one NCCL communicator per distinct device, created here (ranks sharing
+                                       a device use NCCL self send/recv); dist mode: call
+                                       msort_dist_nccl_init on every rank first.  libnccl.so.2 is loaded at
+                                       run time (MSORT_NCCL_LIB overrides); MSORT_ERR_NCCL if unavailable.
+                                       Modes 1 and 4 read each stage's pivots on the host (the NCCL counts
+                                       are host arguments); mode 0 keeps every stage on the GPUs            */
     MSORT_OPT_SKIP_TRIVIAL = 2,  /* 1: skip radix passes whose digit is constant (identity permutation)   */
     MSORT_OPT_HOST_PIPELINE = 3, /* 1 (default): host sorts overlap the transfers with the sort (chunks of
                                        at least 2^20 keys) - the chunk arrives in 4 pieces, each radix sorted
@@ -124,10 +132,16 @@ enum {
                                        back while the next one merges.  msort_dist_sort_host: the merged
                                        chunk enters the merge phase, D2H follows it.  0: H2D, sort, D2H
                                        one after the other                                                */
-    MSORT_OPT_SMALL_GRAPH = 4    /* 1 (default): a one-GPU device sort of <= 2^22 keys repeated on the same
+    MSORT_OPT_SMALL_GRAPH = 4,   /* 1 (default): a one-GPU device sort of <= 2^22 keys repeated on the same
                                        buffer and size replays the whole radix sort as one CUDA graph
                                        (captured on the second call; all passes run, no host round trip on
                                        the histogram); 0: always the launch-by-launch path              */
+    MSORT_OPT_STOP_AFTER_STAGE = 101, /* testing only: end the Alg.2 merge phase (modes 0, 1, 4) after stage
+                                       `value` (-1: all stages); every chunk then holds what the paper's
+                                       stage model holds after that stage (per-stage parity)*/
+    MSORT_OPT_RADIX_EPOCH = 100  /* testing only: set the radix workspace epoch (0..511) so that the next
+                                       sort runs at epoch value+1; the look-back words carry the epoch as a
+                                       tag and the whole workspace is zeroed when it wraps to 0            */
 };
 int msort_set_option(msort_ctx* ctx, int option, int64_t value);
 
@@ -160,6 +174,11 @@ typedef struct {
     double   stage_ms[MSORT_MAX_STAGES];                /* barrier..merge end, max over GPUs       */
     double   stage_exchange_ms[MSORT_MAX_STAGES];       /* merge (fused) or swap+merge kernels     */
     int      kernel_launches;                           /* libmsort kernels launched by this process */
+    int      exchange_mode;                             /* MSORT_OPT_EXCHANGE as run: 0 / 2 fall back to 1 / 3
+                                                           when peer_bulk_ok == 0                      */
+    int      peer_bulk_ok;                              /* 1: TMA bulk copies from peer memory passed the
+                                                           self-test msort_create / msort_dist_import run
+                                                           between distinct devices (or none needed)   */
 } msort_timings;
 
 int msort_get_timings(const msort_ctx* ctx, msort_timings* out);
@@ -247,15 +266,71 @@ int msort_dist_create(msort_ctx** out, int rank, int world, int device, uint64_t
 int msort_dist_export(msort_ctx* ctx, void* handle_out);
 /* Maps every peer's shared buffers from the gathered handles. */
 int msort_dist_import(msort_ctx* ctx, const void* all_handles);
-/* Sort: d_chunk (device pointer on this rank's device, c keys); all ranks call
- * with the same c.  On return rank r holds global ranks [r*c, (r+1)*c).
- * Cross-GPU ordering uses device-side barriers on IPC-mapped flags (timeout ->
- * MSORT_ERR_TIMEOUT).  Blocks until done. */
-int msort_dist_sort(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream);
+/* msort_plan_chunk - the chunking rule ("equally sized chunks",
+ * DESIGN.md reading Q3), host only: for n keys on g GPUs, rank `rank` owns the
+ * input keys [offset, offset + valid) in a chunk of c keys, where
+ *   c      = ceil(n / g) rounded up to a multiple of 4 keys (16-byte alignment),
+ *   offset = min(rank * c, n),   valid = min(max(n - rank * c, 0), c).
+ * The library pads [valid, c) with the largest key under T; the pads sort to
+ * the global end and are dropped, so after a sort rank r's first `valid` keys
+ * are global ranks [offset, offset + valid) of the sorted output.
+ * Outputs may be NULL.  INVALID_ARGUMENT for g not in {1,2,4,8} or rank out of range. */
+int msort_plan_chunk(uint64_t n, int g, int rank, uint64_t* c, uint64_t* offset, uint64_t* valid);
 
-/* End-to-end dist sort: host_keys (this rank's c keys, pinned for full PCIe
- * rate) -> H2D -> msort_dist_sort -> D2H, in place.  Blocks until done. */
-int msort_dist_sort_host(msort_ctx* ctx, void* host_keys, uint64_t c);
+/* msort_dist_sort - device-resident sort of n_total keys spread over the
+ * `world` ranks by msort_plan_chunk: d_chunk (device pointer on this rank's
+ * device, room for c keys, 16-byte aligned) holds this rank's `valid` input
+ * keys; every rank calls with the same n_total.  The library pads the chunk
+ * (reading Q3), sorts, and leaves this rank's `valid` sorted keys (global ranks
+ * [offset, offset + valid)) in d_chunk[0, valid).  Cross-GPU ordering uses
+ * device-side barriers on IPC-mapped flags (timeout -> MSORT_ERR_TIMEOUT).
+ * Ordered after `stream`; blocks until done. */
+int msort_dist_sort(msort_ctx* ctx, void* d_chunk, uint64_t n_total, void* stream);
+
+/* End-to-end dist sort: host_keys holds this rank's `valid` keys
+ * (msort_plan_chunk; pinned for full PCIe rate) -> H2D -> pad -> msort_dist_sort
+ * -> D2H of the `valid` sorted keys, in place.  Blocks until done. */
+int msort_dist_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n_total);
+
+/* Exchange mode 4 in dist mode: rank 0 creates an NCCL unique id
+ * (MSORT_NCCL_ID_BYTES bytes), the caller broadcasts it (e.g. with
+ * torch.distributed), and every rank joins the communicator of `world` ranks.
+ * MSORT_ERR_NCCL on failure (no libnccl, or NCCL refused the ranks - e.g. two
+ * ranks on one GPU). */
+#define MSORT_NCCL_ID_BYTES 128
+int msort_nccl_unique_id(void* out);
+int msort_dist_nccl_init(msort_ctx* ctx, const void* unique_id);
+
+/* ------------------------------------------------------------------------ */
+/* Interconnect peaks (the denominators of the NVLink / PCIe fractions)      */
+/* ------------------------------------------------------------------------ */
+
+typedef struct {
+    double   p2p_ce_gbs;     /* per GPU and direction: mirrored pairs GPU i <-> GPU g-1-i copying concurrently
+                                in both directions (§4.3), copy engines (peer cudaMemcpyAsync) */
+    double   p2p_sm_gbs;     /* same pattern, SM loads through the peer mapping (the fused merge's access)  */
+    double   h2d_gbs;        /* per GPU, all of this context's GPUs copying host->device concurrently (§4.2) */
+    double   d2h_gbs;        /* per GPU, all GPUs device->host concurrently                                  */
+    double   bidir_gbs;      /* per GPU and direction, H2D and D2H at the same time             */
+    uint64_t bytes;          /* bytes per copy (<= one chunk buffer)                                        */
+    int      pairs;          /* mirrored pairs measured (g/2; 0 when g == 1)                                */
+    int      same_device;    /* 1: a pair shares one GPU (virtual ranks): the P2P numbers are HBM copies    */
+} msort_link_peaks;
+
+/* msort_measure_links - time the interconnect patterns above with the
+ * context's own buffers (their contents are overwritten: do not overlap a
+ * sort).  Single process: every rank of the context; the result is the
+ * slowest GPU's rate.  Dist mode: collective (every rank calls it; device
+ * barriers line the ranks up), the result is THIS rank's rate (reduce the
+ * minimum across ranks).  Pinned host buffers of `bytes` per GPU are allocated
+ * and freed inside.  `reps` timed repetitions (mean), after one warm-up. */
+int msort_measure_links(msort_ctx* ctx, uint64_t bytes, int reps, msort_link_peaks* out);
+
+/* msort_release_cached - destroy every context msort_sort cached (device
+ * buffers of about 3 chunk copies per GPU stay allocated between msort_sort
+ * calls otherwise).  Safe to call at any time no msort_sort is running; the
+ * next msort_sort re-creates what it needs. */
+int msort_release_cached(void);
 
 #ifdef __cplusplus
 }

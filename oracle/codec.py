@@ -48,12 +48,3 @@ def decode(codes: np.ndarray, key_type: str) -> np.ndarray:
     dt = {"u32": np.uint32, "u64": np.uint64, "f32": np.float32, "f64": np.float64}[key_type]
     return u.view(dt)
 
-
-def encode_scalar(bits: int, key_type: str) -> int:
-    """T of one key given as its raw bit pattern (pure Python, for Alg.1 walks)."""
-    if key_type not in FLOAT:
-        return bits
-    nb = BITS[key_type]
-    if bits >> (nb - 1):
-        return bits ^ ((1 << nb) - 1)
-    return bits ^ (1 << (nb - 1))

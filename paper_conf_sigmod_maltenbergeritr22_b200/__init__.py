@@ -29,7 +29,9 @@ MSORT_MAX_GPUS = 8
 MSORT_MAX_STAGES = 7
 MSORT_DIST_HANDLE_BYTES = 512
 MSORT_OPT_TIMING, MSORT_OPT_EXCHANGE, MSORT_OPT_SKIP_TRIVIAL, MSORT_OPT_HOST_PIPELINE, MSORT_OPT_SMALL_GRAPH = 0, 1, 2, 3, 4
-EXCHANGE_FUSED, EXCHANGE_SWAP, EXCHANGE_ALLTOALL, EXCHANGE_ALLTOALL_PULL = 0, 1, 2, 3
+MSORT_OPT_RADIX_EPOCH, MSORT_OPT_STOP_AFTER_STAGE = 100, 101  # testing only
+EXCHANGE_FUSED, EXCHANGE_SWAP, EXCHANGE_ALLTOALL, EXCHANGE_ALLTOALL_PULL, EXCHANGE_NCCL = 0, 1, 2, 3, 4
+MSORT_NCCL_ID_BYTES = 128
 MSORT_PASS_ENCODE_IN, MSORT_PASS_DECODE_OUT = 1, 2
 
 STATUS = {0: "MSORT_OK", 1: "MSORT_ERR_INVALID_ARGUMENT", 2: "MSORT_ERR_DEVICE", 3: "MSORT_ERR_OUT_OF_MEMORY",
@@ -42,6 +44,8 @@ EXPORTED = [
     "msort_step_pivot", "msort_merge_workspace_bytes", "msort_step_merge", "msort_step_splitters",
     "msort_plan_num_stages", "msort_plan_stage", "msort_plan_exchange",
     "msort_dist_create", "msort_dist_export", "msort_dist_import", "msort_dist_sort", "msort_dist_sort_host",
+    "msort_plan_chunk", "msort_release_cached", "msort_measure_links", "msort_nccl_unique_id",
+    "msort_dist_nccl_init",
 ]
 
 
@@ -57,7 +61,7 @@ class msort_timings(ctypes.Structure):
         ("stage_keys_exchanged", ctypes.c_uint64 * MSORT_MAX_STAGES),
         ("stage_ms", ctypes.c_double * MSORT_MAX_STAGES),
         ("stage_exchange_ms", ctypes.c_double * MSORT_MAX_STAGES),
-        ("kernel_launches", ctypes.c_int),
+        ("kernel_launches", ctypes.c_int), ("exchange_mode", ctypes.c_int), ("peer_bulk_ok", ctypes.c_int),
     ]
 
     def as_dict(self) -> dict:
@@ -73,8 +77,18 @@ class msort_timings(ctypes.Structure):
             "stage_keys_exchanged": list(self.stage_keys_exchanged[:S]),
             "stage_ms": list(self.stage_ms[:S]),
             "stage_exchange_ms": list(self.stage_exchange_ms[:S]),
-            "kernel_launches": self.kernel_launches,
+            "kernel_launches": self.kernel_launches, "exchange_mode": self.exchange_mode,
+            "peer_bulk_ok": self.peer_bulk_ok,
         }
+
+
+class msort_link_peaks(ctypes.Structure):
+    _fields_ = [("p2p_ce_gbs", ctypes.c_double), ("p2p_sm_gbs", ctypes.c_double), ("h2d_gbs", ctypes.c_double),
+                ("d2h_gbs", ctypes.c_double), ("bidir_gbs", ctypes.c_double), ("bytes", ctypes.c_uint64),
+                ("pairs", ctypes.c_int), ("same_device", ctypes.c_int)]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
 
 
 _P = ctypes.c_void_p
@@ -117,6 +131,11 @@ _sig("msort_dist_export", _I, _P, _P)
 _sig("msort_dist_import", _I, _P, _P)
 _sig("msort_dist_sort", _I, _P, _P, _U64, _P)
 _sig("msort_dist_sort_host", _I, _P, _P, _U64)
+_sig("msort_plan_chunk", _I, _U64, _I, _I, ctypes.POINTER(_U64), ctypes.POINTER(_U64), ctypes.POINTER(_U64))
+_sig("msort_release_cached", _I)
+_sig("msort_measure_links", _I, _P, _U64, _I, ctypes.POINTER(msort_link_peaks))
+_sig("msort_nccl_unique_id", _I, _P)
+_sig("msort_dist_nccl_init", _I, _P, _P)
 
 
 class MsortError(RuntimeError):
@@ -138,8 +157,14 @@ def _kt(key_type) -> int:
 # --- torch plumbing helpers (no compute) ------------------------------------
 
 def key_type_of(t) -> int:
+    """msort key type of a tensor's dtype.  Only unsigned integers and IEEE floats
+    are key types (include/msort.h; reading Q2): a signed tensor would
+    sort its negative values after the positive ones, so it is rejected."""
     import torch
-    m = {torch.uint32: 0, torch.int32: 0, torch.uint64: 1, torch.int64: 1, torch.float32: 2, torch.float64: 3}
+    m = {torch.uint32: 0, torch.uint64: 1, torch.float32: 2, torch.float64: 3}
+    if t.dtype not in m:
+        raise TypeError(f"msort sorts uint32/uint64/float32/float64 keys, not {t.dtype} "
+                        "(signed integers would order negatives after positives)")
     return m[t.dtype]
 
 
@@ -225,6 +250,23 @@ def msort_plan_exchange(g: int, s: int, c: int, pivots: list[int]):
     return list(partner), list(x), list(side)
 
 
+def msort_plan_chunk(n: int, g: int, rank: int) -> tuple[int, int, int]:
+    """(c, offset, valid) of `rank` for n keys on g GPUs (include/msort.h)."""
+    c, off, val = _U64(), _U64(), _U64()
+    _check("msort_plan_chunk", _lib.msort_plan_chunk(n, g, rank, ctypes.byref(c), ctypes.byref(off), ctypes.byref(val)))
+    return c.value, off.value, val.value
+
+
+def msort_nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(MSORT_NCCL_ID_BYTES)
+    _check("msort_nccl_unique_id", _lib.msort_nccl_unique_id(buf))
+    return buf.raw
+
+
+def msort_release_cached() -> None:
+    _check("msort_release_cached", _lib.msort_release_cached())
+
+
 class Context:
     """msort_ctx: pre-allocated buffers/streams/events for g chunks (single process)."""
 
@@ -251,6 +293,11 @@ class Context:
         t = msort_timings()
         _check("msort_get_timings", _lib.msort_get_timings(self._h, ctypes.byref(t)))
         return t.as_dict()
+
+    def measure_links(self, nbytes: int, reps: int = 3) -> dict:
+        pk = msort_link_peaks()
+        _check("msort_measure_links", _lib.msort_measure_links(self._h, nbytes, reps, ctypes.byref(pk)))
+        return pk.as_dict()
 
     def close(self) -> None:
         if getattr(self, "_h", None):
@@ -288,16 +335,30 @@ class DistContext:
     def set_option(self, option: int, value: int) -> None:
         _check("msort_set_option", _lib.msort_set_option(self._h, option, value))
 
-    def sort(self, d_chunk: int, c: int, stream=None) -> None:
-        _check("msort_dist_sort", _lib.msort_dist_sort(self._h, d_chunk, c, stream_ptr(stream)))
+    def nccl_init(self, unique_id: bytes) -> None:
+        """Join the NCCL communicator of all ranks (exchange mode 4); unique_id from rank 0."""
+        if len(unique_id) != MSORT_NCCL_ID_BYTES:
+            raise ValueError("need MSORT_NCCL_ID_BYTES bytes")
+        buf = ctypes.create_string_buffer(unique_id, len(unique_id))
+        _check("msort_dist_nccl_init", _lib.msort_dist_nccl_init(self._h, buf))
 
-    def sort_host(self, host_ptr: int, c: int) -> None:
-        _check("msort_dist_sort_host", _lib.msort_dist_sort_host(self._h, host_ptr, c))
+    def sort(self, d_chunk: int, n_total: int, stream=None) -> None:
+        """d_chunk holds this rank's `valid` keys of the n_total (msort_plan_chunk)."""
+        _check("msort_dist_sort", _lib.msort_dist_sort(self._h, d_chunk, n_total, stream_ptr(stream)))
+
+    def sort_host(self, host_ptr: int, n_total: int) -> None:
+        _check("msort_dist_sort_host", _lib.msort_dist_sort_host(self._h, host_ptr, n_total))
 
     def timings(self) -> dict:
         t = msort_timings()
         _check("msort_get_timings", _lib.msort_get_timings(self._h, ctypes.byref(t)))
         return t.as_dict()
+
+    def measure_links(self, nbytes: int, reps: int = 3) -> dict:
+        """Collective: every rank calls it; this rank's rates."""
+        pk = msort_link_peaks()
+        _check("msort_measure_links", _lib.msort_measure_links(self._h, nbytes, reps, ctypes.byref(pk)))
+        return pk.as_dict()
 
     def close(self) -> None:
         if getattr(self, "_h", None):

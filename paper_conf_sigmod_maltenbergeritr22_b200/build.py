@@ -13,11 +13,27 @@ CSRC = os.path.join(HERE, "csrc")
 INCLUDE = os.path.join(os.path.dirname(HERE), "include")
 BUILD = os.path.join(HERE, "_build")
 LIB = os.path.join(HERE, "libmsort.so")
-SOURCES = ["radix.cu", "merge.cu", "msort.cpp"]
-HEADERS = ["common.cuh", "kernels.h"]
+SOURCES = ["radix.cu", "merge.cu", "msort.cpp", "nccl_shim.cpp"]
+HEADERS = ["common.cuh", "kernels.h", "nccl_shim.h"]
+
+
+def _nccl_include() -> str:
+    """nccl.h for the types of the run-time loaded NCCL (exchange mode 4): torch's NCCL package, else the system."""
+    try:
+        import nvidia.nccl as nn
+        for base in list(getattr(nn, "__path__", [])):
+            inc = os.path.join(base, "include")
+            if os.path.exists(os.path.join(inc, "nccl.h")):
+                return inc
+    except Exception:
+        pass
+    return "/usr/include"
+
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "-I", INCLUDE, "--expt-relaxed-constexpr"]
+FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "-I", INCLUDE, "-I", _nccl_include(),
+         "--expt-relaxed-constexpr"]
+LINK_LIBS = ["-lpthread", "-ldl", "-lrt"]
 
 
 def _nvcc() -> str:
@@ -56,7 +72,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     with ThreadPoolExecutor(len(SOURCES)) as ex:
         objs = list(ex.map(compile_one, SOURCES))
     tmp = LIB + ".tmp"
-    cmd = [nvcc, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs, "-lpthread", "-ldl", "-lrt"]
+    cmd = [nvcc, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs, *LINK_LIBS]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")

@@ -16,16 +16,18 @@ struct RadixWs {
     uint32_t* counters;           // [8] per-pass tile counters
     uint32_t* hist;               // [8][256]
     uint32_t* base;               // [8][256] exclusive digit bases
-    uint32_t* trivial;            // [8] 1 if the pass's digit is constant over all keys; [8..16) largest bin
-    unsigned long long* status;   // [tiles][256] decoupled-lookback words
+    uint32_t* trivial;            // [8] 1 if the pass's digit is constant over all keys; [8..16) largest bin;
+                                  // [16..24) the 4 most frequent digit values of each pass
     unsigned long long* gagg;     // [passes][groups][256] look-back group aggregates (tiles << 32 | sum)
+    unsigned long long* status;   // [tiles][256] decoupled-lookback words (flag << 62 | tag << 32 | count)
     uint64_t tiles;
     uint64_t groups;
     size_t head_bytes;            // bytes of counters..trivial
-    size_t zero_bytes;            // head + status words + group aggregates
-    uint32_t epoch = 0;           // 0: zero the whole workspace and tag status words pass+1; else only the
-                                  // head and the group aggregates are zeroed and status words carry
-                                  // (epoch << 4 | pass+1), so words of earlier sorts never match
+    size_t gagg_bytes;            // bytes of the group aggregates (zeroed per sort, right after the head)
+    size_t zero_bytes;            // head + aggregates + status words for this n
+    size_t alloc_bytes = 0;       // whole workspace allocation (zeroed when a new tag cycle starts, epoch 0)
+    uint32_t epoch = 0;           // 0..511. 0: zero the workspace; status words carry the tag
+                                  // (epoch << 4 | pass + 1), so words of earlier sorts never match
 };
 uint32_t radix_tile_keys(int kt);
 size_t radix_ws_bytes(uint64_t n, int kt);
@@ -40,7 +42,9 @@ cudaError_t launch_histogram(const void* keys, uint64_t n, int kt, uint32_t* his
 cudaError_t launch_scan(const uint32_t* hist, uint32_t* base, uint32_t* trivial, uint64_t n, int kt, cudaStream_t st);
 // true if this GPU serves same-address shared-memory atomics of one warp
 // instruction in lane order (probed once per device; see radix.cu)
-bool atomic_rank_ok();
+// (probed once per device on a private stream; answers false without probing
+// while `caller` or this thread is capturing a CUDA graph)
+bool atomic_rank_ok(cudaStream_t caller = nullptr);
 // one onesweep pass; flags: 1 = encode on load, 2 = decode on store,
 // 4 = atomic ranking (always valid for the first pass; used for every pass when
 // atomic_rank_ok()), 8 = skewed pass: with atomic ranking, the 4 digit values in
@@ -66,6 +70,33 @@ cudaError_t launch_merge(const void* a, uint64_t al, const void* b, uint64_t bl,
 // outputs of merging a and b (a wins ties), j < nparts
 cudaError_t launch_corank(const void* a, uint64_t al, const void* b, uint64_t bl, uint64_t step, uint64_t nparts,
                           int kt, uint64_t* d_part, cudaStream_t st);
+// ----- device-resident Alg.2 stages (exchange mode 0; merge.cu) -----------
+struct BufTable {
+    void* p[8][3];  // [rank][0 = the user chunk, 1 = B0, 2 = B1] (peer pointers for other ranks)
+};
+struct DevStage {   // one replica per rank, in that rank's device memory
+    int32_t cur[8];         // chunk buffer (BufTable slot) holding rank q's current keys
+    uint64_t piv[8][4];     // pivot of group j in stage s (Alg.1)
+};
+struct MergeDesc {  // a two-run merge resolved on the device
+    const void* a;
+    const void* b;
+    void* out;
+    uint64_t al, bl;
+};
+cudaError_t launch_stage_init(DevStage* st, int g, cudaStream_t s);
+cudaError_t launch_stage_pivots(const BufTable& bt, DevStage* st, int stage, int label, int g, uint64_t c, int kt,
+                                cudaStream_t s);
+// resolve this rank's pair exchange -> fused exchange+merge -> rotate every rank's buffer
+cudaError_t launch_stage_merge(const BufTable& bt, DevStage* st, MergeDesc* desc, int stage, int label, int me, int g,
+                               uint64_t c, bool last, int kt, void* mws, cudaStream_t s, int* launches);
+// copy rank me's chunk into the user buffer if the last stage left it in B0/B1
+cudaError_t launch_stage_final(const BufTable& bt, const DevStage* st, int me, uint64_t c, int kt, cudaStream_t s,
+                               int sms);
+
+// SM copy of bytes (multiple of 16, 16-byte aligned; src may be a peer pointer)
+cudaError_t launch_copy_sm(void* dst, const void* src, uint64_t bytes, cudaStream_t st, int sms);
+
 // fill count keys with the largest key under T (tail padding, reading Q3)
 cudaError_t launch_fill_max(void* p, uint64_t count, int kt, cudaStream_t st);
 

@@ -8,7 +8,7 @@
 //                  search of the monotone predicate B[i] < A[|A|-1-i] (reading
 //                  Q5): 7 rounds of 64 parallel remote loads instead of ~2*32
 //                  dependent ones.
-//   partition_kernel / merge_kernel
+//   partition_thread_kernel / merge_pipe_kernel
 //                  the local merge of the two sorted runs a GPU holds after a
 //                  swap as a merge-path merge.  In
 //                  the fused exchange mode run b is the PARTNER's block read over
@@ -173,44 +173,24 @@ __global__ void __launch_bounds__(256) splitter_kernel(GroupPtrs all, int g, uin
     }
 }
 
-template <typename U>
-struct MergeCfg;
-template <>
-struct MergeCfg<uint32_t> {
-    static constexpr int kThreads = 256;
-    static constexpr int kIpt = 15;
-};
-template <>
-struct MergeCfg<uint64_t> {
-    static constexpr int kThreads = 256;
-    static constexpr int kIpt = 7;
-};
-
-// Merge-path partition: part[t] = number of a-elements among the first
-// min(t*TILE, total) outputs (a wins ties).  One warp per boundary.
-template <typename U, bool FLOAT>
-__global__ void __launch_bounds__(128) partition_kernel(const U* __restrict__ a, uint64_t al, const U* __restrict__ b,
-                                                        uint64_t bl, uint64_t tile, uint64_t nparts,
-                                                        uint64_t* __restrict__ part) {
-    const uint64_t w = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
-    if (w >= nparts) return;
-    const uint64_t total = al + bl;
-    const uint64_t k = w * tile < total ? w * tile : total;
-    const uint64_t lo = k > bl ? k - bl : 0;
-    const uint64_t hi = k < al ? k : al;
-    const uint64_t r = warp_first_false(lo, hi, [&](uint64_t i) {
-        return encode<U, FLOAT>(a[i]) <= encode<U, FLOAT>(b[k - 1 - i]);
-    });
-    if ((threadIdx.x & 31) == 0) part[w] = r;
-}
-
 // Same partition, one THREAD per boundary (plain binary search): the top levels
 // of all searches hit the same L2 lines, so DRAM sees only the last few levels
 // of each search (the warp version above touches 64 sectors per round).
+// dyn != nullptr: the runs and their lengths come from device memory (the
+// device-resident Alg.2 stage, resolved on the GPU after the pivot search).
 template <typename U, bool FLOAT>
 __global__ void __launch_bounds__(256) partition_thread_kernel(const U* __restrict__ a, uint64_t al,
                                                                const U* __restrict__ b, uint64_t bl, uint64_t tile,
-                                                               uint64_t nparts, uint64_t* __restrict__ part) {
+                                                               uint64_t nparts, uint64_t* __restrict__ part,
+                                                               const MergeDesc* __restrict__ dyn = nullptr) {
+    if (dyn) {
+        a = static_cast<const U*>(dyn->a);
+        b = static_cast<const U*>(dyn->b);
+        al = dyn->al;
+        bl = dyn->bl;
+        const uint64_t np = (al + bl + tile - 1) / tile + 1;
+        if (np < nparts) nparts = np;
+    }
     const uint64_t w = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
     if (w >= nparts) return;
     const uint64_t total = al + bl;
@@ -225,238 +205,6 @@ __global__ void __launch_bounds__(256) partition_thread_kernel(const U* __restri
     part[w] = lo;
 }
 
-// Block merge of one output tile: stage both input ranges in smem (as codes),
-// per-thread merge-path split, serial merge of IPT outputs, smem transpose,
-// coalesced store.
-template <typename U, bool FLOAT>
-__global__ void __launch_bounds__(MergeCfg<U>::kThreads) merge_kernel(const U* __restrict__ a, const U* __restrict__ b,
-                                                                      uint64_t al, uint64_t bl, U* __restrict__ out,
-                                                                      const uint64_t* __restrict__ part) {
-    constexpr int THREADS = MergeCfg<U>::kThreads;
-    constexpr int IPT = MergeCfg<U>::kIpt;
-    constexpr int TILE = THREADS * IPT;
-    __shared__ U s[TILE];
-    const int tid = threadIdx.x;
-    const uint64_t total = al + bl;
-    const uint64_t k0 = uint64_t(blockIdx.x) * TILE;
-    const uint64_t k1 = k0 + TILE < total ? k0 + TILE : total;
-    const uint64_t a0 = part[blockIdx.x], a1 = part[blockIdx.x + 1];
-    const uint64_t b0 = k0 - a0, b1 = k1 - a1;
-    const int na = int(a1 - a0), nb = int(b1 - b0), nt = na + nb;
-
-    // load: all IPT loads of a thread are independent (in flight together)
-#pragma unroll
-    for (int r = 0; r < IPT; ++r) {
-        const int j = tid + r * THREADS;
-        if (j < nt) s[j] = encode<U, FLOAT>(j < na ? a[a0 + j] : b[b0 + (j - na)]);
-    }
-    __syncthreads();
-    const U* sa = s;
-    const U* sb = s + na;
-    // this thread's output diagonal
-    const int d0 = min(tid * IPT, nt);
-    int lo = max(0, d0 - nb), hi = min(d0, na);
-    while (lo < hi) {
-        const int mid = (lo + hi) >> 1;
-        if (sa[mid] <= sb[d0 - 1 - mid]) lo = mid + 1;
-        else hi = mid;
-    }
-    int ia = lo, ib = d0 - lo;
-    U r[IPT];
-#pragma unroll
-    for (int j = 0; j < IPT; ++j) {
-        const bool takeA = ib >= nb || (ia < na && sa[ia] <= sb[ib]);
-        if (takeA) {
-            r[j] = ia < na ? sa[ia] : U(0);
-            ++ia;
-        } else {
-            r[j] = sb[ib];
-            ++ib;
-        }
-    }
-    __syncthreads();
-#pragma unroll
-    for (int j = 0; j < IPT; ++j)
-        if (d0 + j < nt) s[d0 + j] = r[j];
-    __syncthreads();
-#pragma unroll
-    for (int rr = 0; rr < IPT; ++rr) {
-        const int j = tid + rr * THREADS;
-        if (j < nt) out[k0 + j] = decode<U, FLOAT>(s[j]);
-    }
-}
-
-// ---------------------------------------------------------------------------
-// Persistent merge with bulk (TMA) copies: each block walks its output tiles;
-// while tile i is merged from smem, the A and B input ranges of tile i+1 are
-// already streaming into the other smem stage (cp.async.bulk + mbarrier), and
-// the merged tile leaves through a bulk store.  Input ranges start anywhere:
-// the 16-byte aligned body of each range is bulk-copied, the < 16-byte ragged
-// tail is loaded by threads.  Keys stay raw in smem; comparisons use T(key).
-// ---------------------------------------------------------------------------
-struct MergeMeta {
-    uint64_t a0, b0;       // first input key of the tile in a / b
-    int na, nb;            // keys taken from a / b
-    int headA, headB;      // smem slot of key a0 / b0 inside its region
-    int tailA, tailB;      // first smem slot filled by threads (after the bulk body)
-    int ntailA, ntailB;    // keys loaded by threads
-};
-
-template <typename U>
-struct MergeTmaCfg {
-    static constexpr int kThreads = 256;
-    static constexpr int kIpt = sizeof(U) == 4 ? 15 : 7;
-    static constexpr int kTile = kThreads * kIpt;
-    static constexpr int kV = 16 / int(sizeof(U));
-    static constexpr int kRegion = (kTile + 2 * kV + kV - 1) / kV * kV;  // keys per A or B region
-    static constexpr size_t kSmem = size_t(2) * 2 * kRegion * sizeof(U);
-};
-
-__device__ __forceinline__ void bulk_store_1d(void* dst, const void* src, uint32_t bytes) {
-    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src)),
-                 "r"(bytes)
-                 : "memory");
-    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-}
-
-__device__ __forceinline__ void bulk_wait_read_all() {
-    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
-}
-
-__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
-
-// plan the bulk body / thread tail of one input range [x0, x1) of array `p`
-template <typename U>
-__device__ __forceinline__ uint32_t plan_range(const U* p, uint64_t x0, uint64_t x1, int& head, int& tail,
-                                               int& ntail, const void*& src) {
-    const uintptr_t s = reinterpret_cast<uintptr_t>(p + x0), e = reinterpret_cast<uintptr_t>(p + x1);
-    const uintptr_t as = s & ~uintptr_t(15), ae = e & ~uintptr_t(15);
-    if (x1 <= x0 || ae <= as) {  // no aligned 16-byte unit: everything by threads
-        head = 0;
-        tail = 0;
-        ntail = int(x1 - x0);
-        src = nullptr;
-        return 0;
-    }
-    head = int((s - as) / sizeof(U));
-    tail = int((ae - as) / sizeof(U));
-    ntail = int((e - ae) / sizeof(U));
-    src = reinterpret_cast<const void*>(as);
-    return uint32_t(ae - as);
-}
-
-template <typename U, bool FLOAT>
-__global__ void __launch_bounds__(MergeTmaCfg<U>::kThreads) merge_tma_kernel(const U* __restrict__ a,
-                                                                             const U* __restrict__ b, uint64_t al,
-                                                                             uint64_t bl, U* __restrict__ out,
-                                                                             const uint64_t* __restrict__ part,
-                                                                             uint32_t tiles) {
-    using C = MergeTmaCfg<U>;
-    constexpr int THREADS = C::kThreads, IPT = C::kIpt, TILE = C::kTile, REG = C::kRegion;
-    extern __shared__ __align__(128) unsigned char smem_raw[];
-    U* stage = reinterpret_cast<U*>(smem_raw);  // [2 stages][A region | B region]
-    __shared__ MergeMeta meta[2];
-    __shared__ __align__(8) uint64_t bar[2];
-    const int tid = threadIdx.x;
-    const uint64_t total = al + bl;
-
-    auto issue = [&](uint32_t t, int s) {  // thread 0 only
-        const uint64_t k0 = uint64_t(t) * TILE;
-        const uint64_t k1 = k0 + TILE < total ? k0 + TILE : total;
-        const uint64_t a0 = part[t], a1 = part[t + 1];
-        const uint64_t b0 = k0 - a0, b1 = k1 - a1;
-        MergeMeta& m = meta[s];
-        m.a0 = a0;
-        m.b0 = b0;
-        m.na = int(a1 - a0);
-        m.nb = int(b1 - b0);
-        const void *srcA, *srcB;
-        const uint32_t bytesA = plan_range(a, a0, a1, m.headA, m.tailA, m.ntailA, srcA);
-        const uint32_t bytesB = plan_range(b, b0, b1, m.headB, m.tailB, m.ntailB, srcB);
-        U* dA = stage + size_t(s) * 2 * REG;
-        U* dB = dA + REG;
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&bar[s])),
-                     "r"(bytesA + bytesB)
-                     : "memory");
-        if (bytesA)
-            asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                             smem_u32(dA)),
-                         "l"(srcA), "r"(bytesA), "r"(smem_u32(&bar[s]))
-                         : "memory");
-        if (bytesB)
-            asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                             smem_u32(dB)),
-                         "l"(srcB), "r"(bytesB), "r"(smem_u32(&bar[s]))
-                         : "memory");
-    };
-
-    if (tid == 0) {
-        mbar_init(&bar[0], 1);
-        mbar_init(&bar[1], 1);
-        if (blockIdx.x < tiles) issue(blockIdx.x, 0);
-    }
-    __syncthreads();
-    uint32_t phase[2] = {0, 0};
-    int s = 0;
-    for (uint32_t t = blockIdx.x; t < tiles; t += gridDim.x, s ^= 1) {
-        const uint32_t tn = t + gridDim.x;
-        if (tid == 0 && tn < tiles) {
-            bulk_wait_read_all();  // the other stage's previous bulk store has left smem
-            issue(tn, s ^ 1);
-        }
-        mbar_wait(&bar[s], phase[s]);
-        phase[s] ^= 1;
-        const MergeMeta m = meta[s];
-        U* sA = stage + size_t(s) * 2 * REG;
-        U* sB = sA + REG;
-        if (tid < m.ntailA) sA[m.tailA + tid] = a[m.a0 - m.headA + m.tailA + tid];
-        if (tid >= 32 && tid - 32 < m.ntailB) sB[m.tailB + tid - 32] = b[m.b0 - m.headB + m.tailB + tid - 32];
-        __syncthreads();
-        const U* xa = sA + m.headA;
-        const U* xb = sB + m.headB;
-        const int na = m.na, nb = m.nb, nt = na + nb;
-        const int d0 = min(tid * IPT, nt);
-        int lo = max(0, d0 - nb), hi = min(d0, na);
-        while (lo < hi) {
-            const int mid = (lo + hi) >> 1;
-            if (encode<U, FLOAT>(xa[mid]) <= encode<U, FLOAT>(xb[d0 - 1 - mid])) lo = mid + 1;
-            else hi = mid;
-        }
-        int ia = lo, ib = d0 - lo;
-        U va = ia < na ? xa[ia] : U(0), vb = ib < nb ? xb[ib] : U(0);
-        U r[IPT];
-#pragma unroll
-        for (int j = 0; j < IPT; ++j) {
-            const bool takeA = ib >= nb || (ia < na && encode<U, FLOAT>(va) <= encode<U, FLOAT>(vb));
-            if (takeA) {
-                r[j] = va;
-                ++ia;
-                va = ia < na ? xa[ia] : U(0);
-            } else {
-                r[j] = vb;
-                ++ib;
-                vb = ib < nb ? xb[ib] : U(0);
-            }
-        }
-        __syncthreads();  // every thread is done reading this stage
-#pragma unroll
-        for (int j = 0; j < IPT; ++j)
-            if (d0 + j < nt) sA[d0 + j] = r[j];
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        __syncthreads();
-        U* dst = out + uint64_t(t) * TILE;
-        const bool bulk = ((reinterpret_cast<uintptr_t>(dst) & 15) == 0) && ((uint32_t(nt) * sizeof(U)) % 16 == 0);
-        if (bulk) {
-            if (tid == 0) bulk_store_1d(dst, sA, uint32_t(nt) * sizeof(U));
-        } else {
-            for (int j = tid; j < nt; j += THREADS) dst[j] = sA[j];
-        }
-        __syncthreads();  // scalar readers of this stage done before it is refilled
-    }
-    if (tid == 0) bulk_wait_all();
-}
-
 // ---------------------------------------------------------------------------
 // Deeper pipeline (default): STAGES compact smem stages per block, each holding
 // one output tile's A range followed by its B range (na + nb = TILE keys, plus
@@ -469,6 +217,15 @@ __global__ void __launch_bounds__(MergeTmaCfg<U>::kThreads) merge_tma_kernel(con
 // on the critical path.  A stage is refilled only after the bulk store that
 // read it has finished reading (cp.async.bulk.wait_group.read).
 // ---------------------------------------------------------------------------
+__device__ __forceinline__ void bulk_store_1d(void* dst, const void* src, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src)),
+                 "r"(bytes)
+                 : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
 struct PipeMeta {
     int na, nb;        // keys taken from a / b
     int offA, offB;    // smem slot of key a0 / b0 inside the stage
@@ -488,9 +245,19 @@ struct MergePipeCfg {
 template <typename U, bool FLOAT, int STAGES, int IPT32>
 __global__ void __launch_bounds__(256) merge_pipe_kernel(const U* __restrict__ a, const U* __restrict__ b, uint64_t al,
                                                          uint64_t bl, U* __restrict__ out,
-                                                         const uint64_t* __restrict__ part, uint32_t tiles) {
+                                                         const uint64_t* __restrict__ part, uint32_t tiles,
+                                                         const MergeDesc* __restrict__ dyn) {
     using C = MergePipeCfg<U, STAGES, IPT32>;
     constexpr int THREADS = C::kThreads, IPT = C::kIpt, TILE = C::kTile, SK = C::kStage, V = C::kV;
+    if (dyn) {  // runs resolved on the device (tiles = the launch's upper bound)
+        a = static_cast<const U*>(dyn->a);
+        b = static_cast<const U*>(dyn->b);
+        out = static_cast<U*>(dyn->out);
+        al = dyn->al;
+        bl = dyn->bl;
+        const uint64_t t = (al + bl + TILE - 1) / TILE;
+        if (t < tiles) tiles = uint32_t(t);
+    }
     extern __shared__ __align__(128) unsigned char smem_raw[];
     U* stage = reinterpret_cast<U*>(smem_raw);
     __shared__ PipeMeta meta[STAGES];
@@ -645,24 +412,17 @@ __global__ void __launch_bounds__(256) merge_pipe_kernel(const U* __restrict__ a
     if (tid == 0) bulk_wait_all();
 }
 
-int merge_version() {
-    static int v = -1;
-    if (v < 0) {
-        const char* e = std::getenv("MSORT_MERGE_V");
-        v = e ? std::atoi(e) : 12;  // 12 = the per-key-type default below
-    }
-    return v;
-}
-
+// dyn: the runs come from device memory and al + bl is only an upper bound
 template <typename U, bool FLOAT, int STAGES, int IPT32>
 cudaError_t launch_merge_pipe(const U* a, uint64_t al, const U* b, uint64_t bl, U* out, void* ws, cudaStream_t st,
-                              int* launches) {
+                              int* launches, const MergeDesc* dyn = nullptr) {
     using C = MergePipeCfg<U, STAGES, IPT32>;
     constexpr uint64_t TILE = C::kTile;
     const uint64_t tiles = (al + bl + TILE - 1) / TILE;
     const uint64_t nparts = tiles + 1;
     uint64_t* part = reinterpret_cast<uint64_t*>(ws);
-    partition_thread_kernel<U, FLOAT><<<unsigned((nparts + 255) / 256), 256, 0, st>>>(a, al, b, bl, TILE, nparts, part);
+    partition_thread_kernel<U, FLOAT><<<unsigned((nparts + 255) / 256), 256, 0, st>>>(a, al, b, bl, TILE, nparts, part,
+                                                                                       dyn);
     if (launches) *launches += 2;
     auto kern = merge_pipe_kernel<U, FLOAT, STAGES, IPT32>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(C::kSmem));
@@ -674,52 +434,111 @@ cudaError_t launch_merge_pipe(const U* a, uint64_t al, const U* b, uint64_t bl, 
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     uint64_t grid = uint64_t(per_sm > 0 ? per_sm : 1) * (sms > 0 ? sms : 148);
     if (grid > tiles) grid = tiles;
-    kern<<<unsigned(grid), C::kThreads, C::kSmem, st>>>(a, b, al, bl, out, part, uint32_t(tiles));
+    if (grid == 0) grid = 1;
+    kern<<<unsigned(grid), C::kThreads, C::kSmem, st>>>(a, b, al, bl, out, part, uint32_t(tiles), dyn);
     return cudaGetLastError();
 }
 
+// measured best (profiles/merge_tuning_r1.md): 3 smem stages, 19 keys/thread (u32), 11 (u64)
 template <typename U, bool FLOAT>
 cudaError_t launch_merge_t(const void* a, uint64_t al, const void* b, uint64_t bl, void* out, void* ws,
-                           cudaStream_t st, int* launches) {
-    const U *pa = (const U*)a, *pb = (const U*)b;
-    U* po = (U*)out;
-    switch (merge_version()) {
-        case 0: case 1: case 2: break;  // two-stage kernel below (round-1 reference point)
-        case 4: return launch_merge_pipe<U, FLOAT, 4, 15>(pa, al, pb, bl, po, ws, st, launches);
-        case 5: return launch_merge_pipe<U, FLOAT, 5, 15>(pa, al, pb, bl, po, ws, st, launches);
-        case 6: return launch_merge_pipe<U, FLOAT, 3, 13>(pa, al, pb, bl, po, ws, st, launches);
-        case 7: return launch_merge_pipe<U, FLOAT, 2, 15>(pa, al, pb, bl, po, ws, st, launches);
-        case 8: return launch_merge_pipe<U, FLOAT, 2, 11>(pa, al, pb, bl, po, ws, st, launches);
-        case 9: return launch_merge_pipe<U, FLOAT, 3, 23>(pa, al, pb, bl, po, ws, st, launches);
-        case 10: return launch_merge_pipe<U, FLOAT, 2, 31>(pa, al, pb, bl, po, ws, st, launches);
-        case 11: return launch_merge_pipe<U, FLOAT, 3, 19>(pa, al, pb, bl, po, ws, st, launches);
-        case 3: return launch_merge_pipe<U, FLOAT, 3, 15>(pa, al, pb, bl, po, ws, st, launches);
-        default:  // measured best (profiles/merge_tuning_r1.md): 3 stages, 19 keys/thread (u32), 11 (u64)
-            if constexpr (sizeof(U) == 4) return launch_merge_pipe<U, FLOAT, 3, 19>(pa, al, pb, bl, po, ws, st, launches);
-            else return launch_merge_pipe<U, FLOAT, 3, 23>(pa, al, pb, bl, po, ws, st, launches);
+                           cudaStream_t st, int* launches, const MergeDesc* dyn = nullptr) {
+    constexpr int IPT32 = sizeof(U) == 4 ? 19 : 23;
+    return launch_merge_pipe<U, FLOAT, 3, IPT32>((const U*)a, al, (const U*)b, bl, (U*)out, ws, st, launches, dyn);
+}
+
+// ---------------------------------------------------------------------------
+// Device-resident Alg.2 stage (exchange mode 0): the pivots, every rank's x_d
+// and the chunk-buffer rotation live in device memory (DevStage, one replica
+// per rank), so no stage waits for a host round trip.  Per stage and rank:
+//   stage_pivot_kernel   Alg.1 for every group of the stage (all ranks compute
+//                        all pivots: each replica sees the same values)
+//   stage_resolve_kernel this rank's mirrored-pair exchange (reading Q6) as a
+//                        MergeDesc: own run + partner run (peer pointer) -> the
+//                        other chunk buffer (the user chunk after the last stage)
+//   partition + merge    the fused exchange+merge kernels reading MergeDesc
+//   stage_rotate_kernel  every rank whose x_d != 0 moved to its other buffer
+// and once after the last stage stage_final_kernel copies the chunk into the
+// user buffer if the last stage left it elsewhere (x_d = 0).
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void pair_of(int me, int label, uint64_t c, uint64_t p, int& partner, uint64_t& x,
+                                        int& side) {
+    const int lo = me / label * label, mid = lo + label / 2;
+    const int d = me < mid ? mid - 1 - me : me - mid;
+    partner = me < mid ? mid + d : mid - 1 - d;
+    side = me < mid ? 0 : 1;
+    const uint64_t dc = uint64_t(d) * c;
+    x = p <= dc ? 0 : (p - dc < c ? p - dc : c);
+}
+
+__global__ void stage_init_kernel(DevStage* st, int g) {
+    const int t = threadIdx.x;
+    if (t < 8) st->cur[t] = t < g ? 2 : 0;  // radix output of every rank: B1
+    if (t < 32) (&st->piv[0][0])[t] = 0;
+}
+
+template <typename U, bool FLOAT>
+__global__ void __launch_bounds__(32) stage_pivot_kernel(BufTable bt, DevStage* st, int stage, int label, uint64_t c) {
+    GroupPtrs all;
+#pragma unroll
+    for (int q = 0; q < 8; ++q) all.p[q] = bt.p[q][st->cur[q] & 3];
+    const int half = label / 2;
+    const int first = blockIdx.x * label;
+    const uint64_t s = uint64_t(half) * c;
+    const uint64_t p = warp_first_false(0, s, [&](uint64_t i) {
+        const U b = concat_code<U, FLOAT>(all, first + half, c, i);
+        const U a = concat_code<U, FLOAT>(all, first, c, s - 1 - i);
+        return b < a;
+    });
+    if (threadIdx.x == 0) st->piv[stage][blockIdx.x] = p;
+}
+
+__global__ void stage_resolve_kernel(BufTable bt, const DevStage* st, int stage, int label, int me, uint64_t c,
+                                     int last, int K, MergeDesc* desc) {
+    int partner, side;
+    uint64_t x;
+    pair_of(me, label, c, st->piv[stage][me / label], partner, x, side);
+    MergeDesc m{nullptr, nullptr, nullptr, 0, 0};
+    if (x != 0) {
+        const char* own = static_cast<const char*>(bt.p[me][st->cur[me]]);
+        const char* peer = static_cast<const char*>(bt.p[partner][st->cur[partner]]);
+        m.out = last ? bt.p[me][0] : bt.p[me][st->cur[me] == 1 ? 2 : 1];
+        if (side == 0) {  // L keeps its first c - x keys, receives R's first x
+            m.a = own;
+            m.al = c - x;
+            m.b = peer;
+            m.bl = x;
+        } else {          // R receives L's last x keys, keeps its last c - x
+            m.a = peer + (c - x) * K;
+            m.al = x;
+            m.b = own + x * K;
+            m.bl = c - x;
+        }
     }
-    using C = MergeTmaCfg<U>;
-    constexpr uint64_t TILE = C::kTile;
-    const uint64_t total = al + bl;
-    const uint64_t tiles = (total + TILE - 1) / TILE;
-    const uint64_t nparts = tiles + 1;
-    uint64_t* part = reinterpret_cast<uint64_t*>(ws);
-    const unsigned pblocks = unsigned((nparts * 32 + 127) / 128);
-    partition_kernel<U, FLOAT><<<pblocks, 128, 0, st>>>((const U*)a, al, (const U*)b, bl, TILE, nparts, part);
-    auto kern = merge_tma_kernel<U, FLOAT>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(C::kSmem));
-    if (e != cudaSuccess) return e;
-    int per_sm = 0, dev = 0, sms = 0;
-    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, C::kThreads, C::kSmem)) != cudaSuccess)
-        return e;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    uint64_t grid = uint64_t(per_sm > 0 ? per_sm : 1) * (sms > 0 ? sms : 148);
-    if (grid > tiles) grid = tiles;
-    kern<<<unsigned(grid), C::kThreads, C::kSmem, st>>>((const U*)a, (const U*)b, al, bl, (U*)out, part,
-                                                        uint32_t(tiles));
-    if (launches) *launches += 2;
-    return cudaGetLastError();
+    *desc = m;
+}
+
+__global__ void stage_rotate_kernel(DevStage* st, int stage, int label, int g, uint64_t c, int last) {
+    const int q = threadIdx.x;
+    if (q >= g) return;
+    int partner, side;
+    uint64_t x;
+    pair_of(q, label, c, st->piv[stage][q / label], partner, x, side);
+    const int cur = st->cur[q];
+    __syncwarp();
+    if (x != 0) st->cur[q] = last ? 0 : (cur == 1 ? 2 : 1);
+}
+
+__global__ void stage_final_kernel(BufTable bt, const DevStage* st, int me, uint64_t bytes) {
+    const int cur = st->cur[me];
+    if (cur == 0) return;
+    const uint4* src = static_cast<const uint4*>(bt.p[me][cur]);
+    uint4* dst = static_cast<uint4*>(bt.p[me][0]);
+    const uint64_t n16 = bytes / 16;  // (chunk buffers are 16-byte aligned; a ragged tail follows)
+    for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n16; i += uint64_t(gridDim.x) * blockDim.x)
+        dst[i] = src[i];
+    if (blockIdx.x == 0 && threadIdx.x < bytes % 16)
+        reinterpret_cast<char*>(dst)[n16 * 16 + threadIdx.x] = reinterpret_cast<const char*>(src)[n16 * 16 + threadIdx.x];
 }
 
 template <typename U, bool FLOAT>
@@ -779,9 +598,8 @@ cudaError_t launch_splitters(const GroupPtrs& all, int g, uint64_t c, int kt, ui
 }
 
 size_t merge_ws_bytes(uint64_t total, int kt) {
-    // smallest tile of any merge configuration (MergePipeCfg<.., 11> for the tuning variants)
-    const uint64_t tile = key_bytes(kt) == 4 ? uint64_t(MergePipeCfg<uint32_t, 2, 11>::kTile)
-                                             : uint64_t(MergePipeCfg<uint64_t, 2, 11>::kTile);
+    const uint64_t tile = key_bytes(kt) == 4 ? uint64_t(MergePipeCfg<uint32_t, 3, 19>::kTile)
+                                             : uint64_t(MergePipeCfg<uint64_t, 3, 23>::kTile);
     return size_t((total + tile - 1) / tile + 2) * 8 + 256;
 }
 
@@ -821,6 +639,62 @@ cudaError_t launch_fill_max(void* p, uint64_t count, int kt, cudaStream_t st) {
         case 3: fill_kernel<uint64_t, true><<<blocks, 256, 0, st>>>((uint64_t*)p, count); break;
         default: return cudaErrorInvalidValue;
     }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_stage_init(DevStage* st, int g, cudaStream_t s) {
+    stage_init_kernel<<<1, 32, 0, s>>>(st, g);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_stage_pivots(const BufTable& bt, DevStage* st, int stage, int label, int g, uint64_t c, int kt,
+                                cudaStream_t s) {
+    const int ngroups = g / label;
+    switch (kt) {
+        case 0: stage_pivot_kernel<uint32_t, false><<<ngroups, 32, 0, s>>>(bt, st, stage, label, c); break;
+        case 1: stage_pivot_kernel<uint64_t, false><<<ngroups, 32, 0, s>>>(bt, st, stage, label, c); break;
+        case 2: stage_pivot_kernel<uint32_t, true><<<ngroups, 32, 0, s>>>(bt, st, stage, label, c); break;
+        case 3: stage_pivot_kernel<uint64_t, true><<<ngroups, 32, 0, s>>>(bt, st, stage, label, c); break;
+        default: return cudaErrorInvalidValue;
+    }
+    return cudaGetLastError();
+}
+
+cudaError_t launch_stage_merge(const BufTable& bt, DevStage* st, MergeDesc* desc, int stage, int label, int me, int g,
+                               uint64_t c, bool last, int kt, void* mws, cudaStream_t s, int* launches) {
+    const int K = key_bytes(kt);
+    stage_resolve_kernel<<<1, 1, 0, s>>>(bt, st, stage, label, me, c, last ? 1 : 0, K, desc);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+    // upper bound of the merged length: c (both runs together always hold c keys)
+    const void* dummy = bt.p[me][0];
+    switch (kt) {
+        case 0: e = launch_merge_t<uint32_t, false>(dummy, c, dummy, 0, nullptr, mws, s, launches, desc); break;
+        case 1: e = launch_merge_t<uint64_t, false>(dummy, c, dummy, 0, nullptr, mws, s, launches, desc); break;
+        case 2: e = launch_merge_t<uint32_t, true>(dummy, c, dummy, 0, nullptr, mws, s, launches, desc); break;
+        case 3: e = launch_merge_t<uint64_t, true>(dummy, c, dummy, 0, nullptr, mws, s, launches, desc); break;
+        default: return cudaErrorInvalidValue;
+    }
+    if (e != cudaSuccess) return e;
+    stage_rotate_kernel<<<1, 32, 0, s>>>(st, stage, label, g, c, last ? 1 : 0);
+    if (launches) *launches += 2;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_stage_final(const BufTable& bt, const DevStage* st, int me, uint64_t c, int kt, cudaStream_t s,
+                               int sms) {
+    stage_final_kernel<<<unsigned(sms > 0 ? sms * 4 : 592), 256, 0, s>>>(bt, st, me, c * uint64_t(key_bytes(kt)));
+    return cudaGetLastError();
+}
+
+__global__ void __launch_bounds__(256) copy16_kernel(uint4* __restrict__ dst, const uint4* __restrict__ src, uint64_t n16) {
+    for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n16; i += uint64_t(gridDim.x) * blockDim.x)
+        dst[i] = __ldcs(src + i);
+}
+
+cudaError_t launch_copy_sm(void* dst, const void* src, uint64_t bytes, cudaStream_t st, int sms) {
+    copy16_kernel<<<unsigned(sms > 0 ? sms * 8 : 1184), 256, 0, st>>>(static_cast<uint4*>(dst),
+                                                                      static_cast<const uint4*>(src), bytes / 16);
     return cudaGetLastError();
 }
 

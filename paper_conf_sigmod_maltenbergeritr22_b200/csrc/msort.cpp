@@ -30,6 +30,7 @@
 
 #include "../../include/msort.h"
 #include "kernels.h"
+#include "nccl_shim.h"
 
 using namespace msort;
 
@@ -127,6 +128,7 @@ uint64_t chunk_size(uint64_t n, int g) {
 // ---------------------------------------------------------------------------
 constexpr int kPieces = 4;   // pipelined host sort: H2D pieces, each sorted while the next one arrives
 constexpr int kSlices = 4;   // ... and final-merge slices, each copied back while the next one merges
+constexpr uint32_t kEpochs = 512;  // radix tag cycle (RadixWs::epoch)
 
 struct Rank {
     int dev = 0;
@@ -140,6 +142,9 @@ struct Rank {
     uint64_t* d_pivot = nullptr;   // [128] pivots (Alg.2) or splitters (all-to-all)
     uint64_t* h_pivot = nullptr;   // pinned [128]
     uint32_t* h_trivial = nullptr; // pinned [24]: trivial flags, largest bin per pass, its digit
+    DevStage* d_stage = nullptr;   // device-resident Alg.2 state (exchange mode 0): buffer rotation, pivots
+    DevStage* h_stage = nullptr;   // pinned copy read after the sort (stage statistics)
+    MergeDesc* d_desc = nullptr;   // this rank's exchange+merge of the current stage, resolved on the GPU
     int* d_err = nullptr;          // barrier timeout flag
     int* h_err = nullptr;          // pinned
     cudaEvent_t e_begin = nullptr, e_hist = nullptr, e_sorted = nullptr, e_end = nullptr;
@@ -158,6 +163,7 @@ struct Rank {
     int small_timing = -1;
     bool small_seen = false;
     cudaEvent_t e_sync[MSORT_MAX_STAGES + 1] = {};
+    cudaEvent_t e_nccl[2] = {};  // exchange mode 4: ranks sharing a device hand their stream to one NCCL stream
     cudaEvent_t e_stage[MSORT_MAX_STAGES][2] = {};
     cudaEvent_t e_xch[MSORT_MAX_STAGES][2] = {};
     bool xch_rec[MSORT_MAX_STAGES] = {};  // e_xch[s] recorded in this sort
@@ -167,8 +173,9 @@ struct Rank {
     int passes_run = 0;
     int pass_ids[8] = {};
     // radix workspace epoch (RadixWs::epoch); starts so that the first sort
-    // zeroes the whole workspace, and wraps to 0 (full zeroing) every 2^26 sorts
-    uint32_t radix_epoch = (1u << 26) - 1;
+    // zeroes the whole workspace, and wraps to 0 (the whole allocation zeroed
+    // again) every kEpochs sorts
+    uint32_t radix_epoch = kEpochs - 1;
 
     void* ptr(int which) const { return which < 0 ? user : buf[which]; }
 };
@@ -198,19 +205,33 @@ struct msort_ctx {
     std::vector<void*> opened;
     // options
     int timing = 1;
-    int exchange = 0;
+    int exchange = 0;       // MSORT_OPT_EXCHANGE as requested
+    int xmode = 0;          // as run: 0 / 2 fall back to 1 / 3 when bulk copies from peer memory failed the
+                            // self-test (peer_bulk_ok)
+    bool peer_bulk_ok = true;
     int skip_trivial = 1;
     int host_pipeline = 1;
     int small_graph = 1;
+    bool stats_on_device = false;  // the sort's stage statistics are in r[0].h_stage (device-resident Alg.2)
+    // exchange mode 4 (NCCL send/recv swap): single process - one comm per distinct device (ncclCommInitAll),
+    // rank i uses comm nccl_comm[i] with comm rank nccl_rank[i]; dist - one comm of `g` ranks
+    int stop_after = -1;  // testing (MSORT_OPT_STOP_AFTER_STAGE): end the Alg.2 merge phase after this stage
+    NcclState nccl;
+    int nccl_comm[MSORT_MAX_GPUS] = {};
+    int nccl_rank[MSORT_MAX_GPUS] = {};
     msort_timings tm{};
 };
 
 namespace {
 
+int stages_to_run(const msort_ctx* ctx, int S) {
+    return ctx->stop_after >= 0 ? std::min(S, ctx->stop_after + 1) : S;
+}
+
 int alloc_rank(msort_ctx* ctx, Rank& R, bool need_b1, bool need_stage) {
     const size_t K = key_bytes(ctx->kt);
     CUDA_TRY(cudaSetDevice(R.dev));
-    atomic_rank_ok();  // one-time per-device probe, outside any sort
+    atomic_rank_ok(nullptr);  // one-time per-device probe, outside any sort
     CUDA_TRY(cudaStreamCreateWithFlags(&R.st, cudaStreamNonBlocking));
     CUDA_TRY(cudaStreamCreateWithFlags(&R.cst, cudaStreamNonBlocking));
     for (auto& e : R.e_piece) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
@@ -227,6 +248,9 @@ int alloc_rank(msort_ctx* ctx, Rank& R, bool need_b1, bool need_stage) {
     CUDA_TRY(cudaMalloc(&R.d_pivot, 128 * sizeof(uint64_t)));
     CUDA_TRY(cudaMalloc(&R.d_err, sizeof(int)));
     CUDA_TRY(cudaMemset(R.d_err, 0, sizeof(int)));
+    CUDA_TRY(cudaMalloc(&R.d_stage, sizeof(DevStage)));
+    CUDA_TRY(cudaMalloc(&R.d_desc, sizeof(MergeDesc)));
+    CUDA_TRY(cudaMallocHost(&R.h_stage, sizeof(DevStage)));
     CUDA_TRY(cudaMallocHost(&R.h_pivot, 128 * sizeof(uint64_t)));
     CUDA_TRY(cudaMallocHost(&R.h_trivial, 24 * sizeof(uint32_t)));
     CUDA_TRY(cudaMallocHost(&R.h_err, sizeof(int)));
@@ -236,6 +260,7 @@ int alloc_rank(msort_ctx* ctx, Rank& R, bool need_b1, bool need_stage) {
     for (auto& pe : R.e_pass)
         for (auto& e : pe) CUDA_TRY(cudaEventCreate(&e));
     for (auto& e : R.e_sync) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    for (auto& e : R.e_nccl) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     for (auto& se : R.e_stage)
         for (auto& e : se) CUDA_TRY(cudaEventCreate(&e));
     for (auto& xe : R.e_xch)
@@ -254,6 +279,9 @@ void free_rank(Rank& R) {
     if (R.mws) cudaFree(R.mws);
     if (R.d_pivot) cudaFree(R.d_pivot);
     if (R.d_err) cudaFree(R.d_err);
+    if (R.d_stage) cudaFree(R.d_stage);
+    if (R.d_desc) cudaFree(R.d_desc);
+    if (R.h_stage) cudaFreeHost(R.h_stage);
     if (R.h_pivot) cudaFreeHost(R.h_pivot);
     if (R.h_trivial) cudaFreeHost(R.h_trivial);
     if (R.h_err) cudaFreeHost(R.h_err);
@@ -264,6 +292,8 @@ void free_rank(Rank& R) {
         for (auto e : pe)
             if (e) cudaEventDestroy(e);
     for (auto e : R.e_sync)
+        if (e) cudaEventDestroy(e);
+    for (auto e : R.e_nccl)
         if (e) cudaEventDestroy(e);
     for (auto& se : R.e_stage)
         for (auto e : se)
@@ -299,8 +329,9 @@ float elapsed(cudaEvent_t a, cudaEvent_t b) {
 int radix_begin(msort_ctx* ctx, Rank& R, const void* src, uint64_t c) {
     CUDA_TRY(cudaSetDevice(R.dev));
     RadixWs ws = radix_ws_layout(R.rws, c, ctx->kt);
-    R.radix_epoch = (R.radix_epoch + 1) & ((1u << 26) - 1);
+    R.radix_epoch = (R.radix_epoch + 1) % kEpochs;
     ws.epoch = R.radix_epoch;
+    ws.alloc_bytes = R.rws_bytes;
     CUDA_TRY(radix_prologue(src, c, ctx->kt, ws, R.st));
     ctx->tm.kernel_launches += 2;
     if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_hist, R.st));
@@ -370,7 +401,7 @@ int radix_passes(msort_ctx* ctx, Rank& R, const void* src, void* dst, void* tmp,
         const bool skewed = maxbin * 16 > c;
         const int mode = skew_mode();
         const bool dominant = mode == 1 ? skewed : (mode == 0 ? false : maxbin * 4 > c);
-        bool atomic_rank = j == 0 || atomic_rank_ok();
+        bool atomic_rank = j == 0 || atomic_rank_ok(R.st);
         if (skewed && !dominant) atomic_rank = false;  // peer match
         const bool hot = dominant && atomic_rank;
         const int flags = (j == 0 ? 1 : 0) | (j == E - 1 ? 2 : 0) | (atomic_rank ? 4 : 0) | (hot ? 8 : 0);
@@ -396,11 +427,20 @@ int launch_exchange(msort_ctx* ctx, Rank& R, int stage, bool last, uint64_t c, u
     if (x == 0) return MSORT_OK;  // Alg.2 line 7 / reading Q8
     const int out_idx = last ? -1 : (R.cur == 0 ? 1 : 0);
     void* out = R.ptr(out_idx);
-    if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[stage][0], R.st));
+    // (mode 4 recorded the start before the NCCL swap)
+    if (ctx->timing && ctx->xmode != 4) CUDA_TRY(cudaEventRecord(R.e_xch[stage][0], R.st));
     if (x == c) {
-        // the whole chunk moves: a pure P2P copy (one sorted run, reading Q8)
-        CUDA_TRY(cudaMemcpyAsync(out, peer, c * K, cudaMemcpyDefault, R.st));
-    } else if (ctx->exchange == 0) {
+        // the whole chunk moves: a pure P2P copy (one sorted run, reading Q8);
+        // mode 4 received it into `out` already
+        if (ctx->xmode != 4) CUDA_TRY(cudaMemcpyAsync(out, peer, c * K, cudaMemcpyDefault, R.st));
+    } else if (ctx->xmode == 4) {
+        // NCCL swap done (nccl_stage_exchange): the partner's block is in B2
+        const char* recv = static_cast<const char*>(R.buf[2]);
+        if (side == 0)
+            CUDA_TRY(launch_merge(ownb, c - x, recv, x, out, ctx->kt, R.mws, R.st, &ctx->tm.kernel_launches));
+        else
+            CUDA_TRY(launch_merge(recv, x, ownb + x * K, c - x, out, ctx->kt, R.mws, R.st, &ctx->tm.kernel_launches));
+    } else if (ctx->xmode == 0) {
         // fused: the merge kernel reads the partner's block over NVLink
         if (side == 0)
             CUDA_TRY(launch_merge(ownb, c - x, peerb, x, out, ctx->kt, R.mws, R.st, &ctx->tm.kernel_launches));
@@ -423,14 +463,196 @@ int launch_exchange(msort_ctx* ctx, Rank& R, int stage, bool last, uint64_t c, u
     return MSORT_OK;
 }
 
+// --- exchange mode 4: the swap as NCCL send/recv (S5, north_star) -----------------
+
+// Single process: one communicator per distinct device of the context
+// (ncclCommInitAll); ranks sharing a device (virtual ranks) share its comm and
+// exchange through NCCL's self send/recv.
+int nccl_init_local(msort_ctx* ctx) {
+    std::vector<int> devs;
+    for (int i = 0; i < ctx->g; ++i) {
+        const int d = ctx->r[i].dev;
+        int idx = -1;
+        for (int u = 0; u < int(devs.size()); ++u)
+            if (devs[u] == d) idx = u;
+        if (idx < 0) {
+            idx = int(devs.size());
+            devs.push_back(d);
+        }
+        ctx->nccl_comm[i] = idx;
+        ctx->nccl_rank[i] = idx;
+    }
+    std::string err;
+    DeviceGuard guard;
+    if (!nccl_init_all(ctx->nccl, devs.data(), int(devs.size()), &err)) return set_error(MSORT_ERR_NCCL, err);
+    return MSORT_OK;
+}
+
+// Post one stage's swap for the ranks this process drives: every rank with
+// x != 0 sends its outgoing block (L: its last x keys, R: its first x keys,
+// reading Q6) to its partner and receives the partner's block into its receive
+// buffer B2 - or, when the whole chunk moves (x == c), straight into the
+// buffer the stage writes.  Sends are posted in rank order, then the receives
+// in the order of their senders, so matching pairs line up per comm pair.
+// Ranks on one device run their NCCL calls on the first such rank's stream.
+int nccl_stage_exchange(msort_ctx* ctx, const Exchange& ex, uint64_t c, bool last) {
+    const size_t K = key_bytes(ctx->kt);
+    const int nl = ctx->nlocal;
+    auto me_of = [&](int i) { return ctx->dist ? ctx->rank : i; };
+    auto lead_of = [&](int i) {
+        for (int q = 0; q < nl; ++q)
+            if (ctx->r[q].dev == ctx->r[i].dev) return q;
+        return i;
+    };
+    // hand every rank's stream to its device's NCCL stream
+    for (int i = 0; i < nl; ++i) {
+        const int l = lead_of(i);
+        if (l == i) continue;
+        CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
+        CUDA_TRY(cudaEventRecord(ctx->r[i].e_nccl[0], ctx->r[i].st));
+        CUDA_TRY(cudaStreamWaitEvent(ctx->r[l].st, ctx->r[i].e_nccl[0], 0));
+    }
+    std::vector<P2POp> ops;
+    for (int i = 0; i < nl; ++i) {  // sends
+        const int me = me_of(i);
+        const uint64_t x = ex.x[me];
+        if (x == 0) continue;
+        const Rank& R = ctx->r[i];
+        const char* own = static_cast<const char*>(R.ptr(R.cur));
+        const int partner = ex.partner[me];
+        const int peer_rank = ctx->dist ? partner : ctx->nccl_rank[partner];
+        ops.push_back({true, own + (ex.side[me] == 0 ? (c - x) : 0) * K, x * K, peer_rank,
+                       ctx->dist ? 0 : ctx->nccl_comm[i], ctx->r[lead_of(i)].st});
+    }
+    for (int sidx = 0; sidx < ctx->g; ++sidx) {  // receives, in the order of their senders
+        const int recv_me = ex.partner[sidx];
+        if (recv_me < 0 || ex.x[sidx] == 0) continue;
+        int i = -1;  // local index of the receiving rank
+        if (ctx->dist) {
+            if (recv_me == ctx->rank) i = 0;
+        } else {
+            i = recv_me;
+        }
+        if (i < 0) continue;
+        if (ctx->dist && ctx->rank != recv_me) continue;
+        Rank& R = ctx->r[i];
+        const uint64_t x = ex.x[recv_me];
+        void* dst = x == c ? R.ptr(last ? -1 : (R.cur == 0 ? 1 : 0)) : R.buf[2];
+        const int peer_rank = ctx->dist ? sidx : ctx->nccl_rank[sidx];
+        ops.push_back({false, dst, x * K, peer_rank, ctx->dist ? 0 : ctx->nccl_comm[i], ctx->r[lead_of(i)].st});
+    }
+    std::string err;
+    {
+        DeviceGuard guard;
+        if (!ops.empty() && !nccl_group(ctx->nccl, ops, &err)) return set_error(MSORT_ERR_NCCL, err);
+    }
+    for (int i = 0; i < nl; ++i) {
+        const int l = lead_of(i);
+        if (l == i) continue;
+        CUDA_TRY(cudaSetDevice(ctx->r[l].dev));
+        CUDA_TRY(cudaEventRecord(ctx->r[l].e_nccl[1], ctx->r[l].st));
+        CUDA_TRY(cudaStreamWaitEvent(ctx->r[i].st, ctx->r[l].e_nccl[1], 0));
+    }
+    return MSORT_OK;
+}
+
+// --- exchange mode actually run ----------------------------------------------------
+
+// The fused modes (0: Alg.2 merge reading the partner's block, 2: NEXT-1 merge
+// reading the runs) move peer memory with TMA bulk copies (cp.async.bulk) in
+// merge_pipe_kernel; if the self-test below found that this does not work
+// between two of the context's GPUs, they fall back to the copy-engine modes
+// 1 / 3 (peer copy into a local buffer, then a local merge).
+int apply_exchange_mode(msort_ctx* ctx) {
+    int m = ctx->exchange;
+    if (!ctx->peer_bulk_ok) m = m == 0 ? 1 : (m == 2 ? 3 : m);
+    if (m == 1 || m == 4)
+        for (int i = 0; i < ctx->nlocal; ++i)
+            if (!ctx->r[i].buf[2]) {
+                CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
+                CUDA_TRY(cudaMalloc(&ctx->r[i].buf[2], std::max<size_t>(ctx->cap * key_bytes(ctx->kt), 256)));
+            }
+    ctx->xmode = m;
+    return MSORT_OK;
+}
+
+// Self-test of the fused exchange's access path: a merge on GPU `me` whose
+// second run lives in a peer's buffer (read by cp.async.bulk through the peer
+// mapping, starting one key past a 16-byte boundary) must equal the merge of
+// the known patterns.  a: local even keys, b: peer odd keys.
+constexpr uint32_t kSelfTestKeys = 4099;
+
+void selftest_pattern(std::vector<uint32_t>& even, std::vector<uint32_t>& odd, uint32_t n) {
+    even.resize(n);
+    odd.resize(n);
+    for (uint32_t k = 0; k < n; ++k) {
+        even[k] = 2 * k;
+        odd[k] = 2 * k + 1;
+    }
+}
+
+// merge local even[0..n) with peer_odd[1..n) on rank R; true if the result is right
+int selftest_merge(msort_ctx* ctx, Rank& R, const void* peer_odd, uint32_t n, bool* ok) {
+    std::vector<uint32_t> even, odd, got(2 * n - 1);
+    selftest_pattern(even, odd, n);
+    CUDA_TRY(cudaSetDevice(R.dev));
+    CUDA_TRY(cudaMemcpyAsync(R.stage, even.data(), n * 4, cudaMemcpyHostToDevice, R.st));
+    CUDA_TRY(launch_merge(R.stage, n, static_cast<const uint32_t*>(peer_odd) + 1, n - 1, R.buf[1], 0, R.mws, R.st,
+                          nullptr));
+    CUDA_TRY(cudaMemcpyAsync(got.data(), R.buf[1], (2 * n - 1) * 4, cudaMemcpyDeviceToHost, R.st));
+    CUDA_TRY(cudaStreamSynchronize(R.st));
+    bool good = true;
+    for (uint32_t k = 0, t = 0; k < 2 * n - 1; ++k) {  // expected: 0, 2, 3, 4, 5, ... (odd 1 skipped)
+        const uint32_t want = k == 0 ? 0 : k + 1;
+        good = good && got[k] == want;
+        (void)t;
+    }
+    *ok = good;
+    return MSORT_OK;
+}
+
+int peer_bulk_selftest_local(msort_ctx* ctx) {
+    const uint32_t n = kSelfTestKeys;
+    if (ctx->cap < 2 * uint64_t(n)) return MSORT_OK;  // (tiny contexts: nothing to test with)
+    std::vector<uint32_t> even, odd;
+    selftest_pattern(even, odd, n);
+    bool tested[MSORT_MAX_GPUS][MSORT_MAX_GPUS] = {};
+    for (int i = 0; i < ctx->g; ++i)
+        for (int j = 0; j < ctx->g; ++j) {
+            Rank &A = ctx->r[i], &B = ctx->r[j];
+            if (A.dev == B.dev || tested[i][j]) continue;
+            for (int a = 0; a < ctx->g; ++a)
+                for (int b = 0; b < ctx->g; ++b)
+                    if (ctx->r[a].dev == A.dev && ctx->r[b].dev == B.dev) tested[a][b] = true;
+            CUDA_TRY(cudaSetDevice(B.dev));
+            CUDA_TRY(cudaMemcpy(B.buf[0], odd.data(), n * 4, cudaMemcpyHostToDevice));
+            bool ok = false;
+            const int st = selftest_merge(ctx, A, B.buf[0], n, &ok);
+            if (st != MSORT_OK || !ok) ctx->peer_bulk_ok = false;
+        }
+    return MSORT_OK;
+}
+
 int check_c(msort_ctx* ctx, uint64_t c) {
     if (c > ctx->cap) return set_error(MSORT_ERR_INVALID_ARGUMENT, "keys per GPU exceed the context capacity");
     if (c >= (1ull << 32)) return set_error(MSORT_ERR_INVALID_ARGUMENT, "keys per GPU must be < 2^32");
     return MSORT_OK;
 }
 
+int sm_count_of(int dev) {
+    int n = 0;
+    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) {
+        cudaGetLastError();
+        return 148;
+    }
+    return n > 0 ? n : 148;
+}
+
 void reset_timings(msort_ctx* ctx, uint64_t c) {
+    ctx->stats_on_device = false;
     ctx->tm = msort_timings{};
+    ctx->tm.exchange_mode = ctx->xmode;
+    ctx->tm.peer_bulk_ok = ctx->peer_bulk_ok ? 1 : 0;
     ctx->tm.n_gpus = ctx->g;
     ctx->tm.keys_per_gpu = c;
     ctx->tm.passes_total = num_passes(ctx->kt);
@@ -568,7 +790,7 @@ int alltoall_local(msort_ctx* ctx, uint64_t c) {
     CUDA_TRY(cudaStreamSynchronize(R0.st));
     std::vector<uint64_t> s(R0.h_pivot, R0.h_pivot + (g + 1) * g);
     record_alltoall_stats(ctx, s.data(), g);
-    if (ctx->exchange == 2) {
+    if (ctx->xmode == 2) {
         // fused: every rank merges its runs straight out of the peers' B1
         for (int j = 0; j < g; ++j) {
             Rank& R = ctx->r[j];
@@ -649,7 +871,7 @@ int capture_small(msort_ctx* ctx, Rank& R, uint64_t c) {
         for (int p = 0; p < P; ++p) {
             const void* in = (p % 2 == 0) ? R.user : R.buf[0];
             void* out = (p % 2 == 0) ? R.buf[0] : R.user;
-            const int flags = (p == 0 ? 1 : 0) | (p == P - 1 ? 2 : 0) | ((p == 0 || atomic_rank_ok()) ? 4 : 0);
+            const int flags = (p == 0 ? 1 : 0) | (p == P - 1 ? 2 : 0) | ((p == 0 || atomic_rank_ok(R.st)) ? 4 : 0);
             if (ctx->timing) CUDA_TRY(rec(R.e_pass[p][0]));
             CUDA_TRY(launch_onesweep(in, out, c, ctx->kt, p, flags, ws, ws.base + p * 256, R.st));
             if (ctx->timing) CUDA_TRY(rec(R.e_pass[p][1]));
@@ -695,6 +917,69 @@ int sort_small_graph(msort_ctx* ctx, Rank& R, uint64_t c, bool* done) {
     return MSORT_OK;
 }
 
+// Alg.2 merge phase with every decision on the GPUs (exchange mode 0): per
+// stage an event barrier across the ranks' streams, then on every rank the
+// pivots of all groups (Alg.1), this rank's fused exchange+merge resolved from
+// them, and the buffer rotation of all ranks - no host round trip until the
+// sort ends.  Ranks start from B1 (the radix output, R.cur == 1).
+int alg2_device_local(msort_ctx* ctx, uint64_t c) {
+    const int g = ctx->g;
+    std::vector<int> labels;
+    stage_labels(g, labels);
+    const int S = int(labels.size());
+    BufTable bt{};
+    for (int q = 0; q < g; ++q) {
+        bt.p[q][0] = ctx->r[q].user;
+        bt.p[q][1] = ctx->r[q].buf[0];
+        bt.p[q][2] = ctx->r[q].buf[1];
+    }
+    for (int i = 0; i < g; ++i) {
+        Rank& R = ctx->r[i];
+        CUDA_TRY(cudaSetDevice(R.dev));
+        CUDA_TRY(launch_stage_init(R.d_stage, g, R.st));
+        ctx->tm.kernel_launches += 1;
+    }
+    const int S_run = stages_to_run(ctx, S);
+    ctx->tm.n_stages = S_run;
+    for (int s = 0; s < S_run; ++s) {
+        const int label = labels[s];
+        const bool last = s == S - 1;
+        // barrier: every rank's stream waits for every other rank's previous stage
+        for (int i = 0; i < g; ++i) {
+            CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
+            CUDA_TRY(cudaEventRecord(ctx->r[i].e_sync[s], ctx->r[i].st));
+        }
+        for (int i = 0; i < g; ++i) {
+            Rank& R = ctx->r[i];
+            CUDA_TRY(cudaSetDevice(R.dev));
+            for (int q = 0; q < g; ++q)
+                if (q != i) CUDA_TRY(cudaStreamWaitEvent(R.st, ctx->r[q].e_sync[s], 0));
+            if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[s][0], R.st));
+            CUDA_TRY(launch_stage_pivots(bt, R.d_stage, s, label, g, c, ctx->kt, R.st));
+            ctx->tm.kernel_launches += 1;
+            if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[s][0], R.st));
+            CUDA_TRY(launch_stage_merge(bt, R.d_stage, R.d_desc, s, label, i, g, c, last, ctx->kt, R.mws, R.st,
+                                        &ctx->tm.kernel_launches));
+            if (ctx->timing) {
+                CUDA_TRY(cudaEventRecord(R.e_xch[s][1], R.st));
+                R.xch_rec[s] = true;
+                CUDA_TRY(cudaEventRecord(R.e_stage[s][1], R.st));
+            }
+        }
+    }
+    for (int i = 0; i < g; ++i) {
+        Rank& R = ctx->r[i];
+        CUDA_TRY(cudaSetDevice(R.dev));
+        CUDA_TRY(launch_stage_final(bt, R.d_stage, i, c, ctx->kt, R.st, sm_count_of(R.dev)));
+        ctx->tm.kernel_launches += 1;
+        if (i == 0) CUDA_TRY(cudaMemcpyAsync(R.h_stage, R.d_stage, sizeof(DevStage), cudaMemcpyDeviceToHost, R.st));
+        R.cur = -1;
+        CUDA_TRY(cudaEventRecord(R.e_end, R.st));
+    }
+    ctx->stats_on_device = true;
+    return MSORT_OK;
+}
+
 int sort_device_local(msort_ctx* ctx, uint64_t c) {
     const int g = ctx->g;
     if (g == 1 && c <= kGraphMaxKeys && ctx->small_graph) {
@@ -724,10 +1009,12 @@ int sort_device_local(msort_ctx* ctx, uint64_t c) {
         }
         CUDA_TRY(cudaEventRecord(R.e_sorted, R.st));
     }
-    if (g > 1 && ctx->exchange >= 2) return alltoall_local(ctx, c);
+    if (g > 1 && (ctx->xmode == 2 || ctx->xmode == 3)) return alltoall_local(ctx, c);
+    if (g > 1 && ctx->xmode == 0) return alg2_device_local(ctx, c);
     const int S = int(labels.size());
-    ctx->tm.n_stages = S;
-    for (int s = 0; s < S; ++s) {
+    const int S_run = stages_to_run(ctx, S);
+    ctx->tm.n_stages = S_run;
+    for (int s = 0; s < S_run; ++s) {
         const int label = labels[s];
         const bool last = s == S - 1;
         // barrier: every rank's stream waits for every other rank's previous stage
@@ -765,6 +1052,14 @@ int sort_device_local(msort_ctx* ctx, uint64_t c) {
         }
         ctx->tm.stage_max_x[s] = mx;
         ctx->tm.stage_keys_exchanged[s] = sum;
+        if (ctx->xmode == 4) {  // S5 as NCCL send/recv, then S6 below
+            for (int i = 0; i < g; ++i)
+                if (ctx->timing && ex.x[i]) {
+                    CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
+                    CUDA_TRY(cudaEventRecord(ctx->r[i].e_xch[s][0], ctx->r[i].st));
+                }
+            MSORT_TRY(nccl_stage_exchange(ctx, ex, c, last));
+        }
         // S5+S6 on every rank
         int new_cur[MSORT_MAX_GPUS];
         for (int i = 0; i < g; ++i) {
@@ -785,6 +1080,31 @@ int sort_device_local(msort_ctx* ctx, uint64_t c) {
         CUDA_TRY(cudaEventRecord(R.e_end, R.st));
     }
     return MSORT_OK;
+}
+
+// Stage statistics of a device-resident Alg.2 merge phase from the pivots the
+// GPUs computed (h_stage, copied back with the sort's last D2H).
+void stage_stats_from_device(msort_ctx* ctx, const DevStage& ds, uint64_t c) {
+    std::vector<int> labels;
+    stage_labels(ctx->g, labels);
+    const int S = stages_to_run(ctx, int(labels.size()));
+    ctx->tm.n_stages = S;
+    for (int s = 0; s < S; ++s) {
+        const int label = labels[s], ngroups = ctx->g / label;
+        uint64_t piv[MSORT_MAX_GPUS / 2] = {};
+        for (int j = 0; j < ngroups; ++j) piv[j] = ds.piv[s][j];
+        Exchange ex;
+        plan_exchange(ctx->g, label, c, piv, ex);
+        ctx->tm.stage_label[s] = label;
+        uint64_t mx = 0, sum = 0;
+        for (int j = 0; j < ngroups; ++j) ctx->tm.stage_pivot[s][j] = piv[j];
+        for (int q = 0; q < ctx->g; ++q) {
+            mx = std::max(mx, ex.x[q]);
+            if (ex.side[q] == 0) sum += ex.x[q];
+        }
+        ctx->tm.stage_max_x[s] = mx;
+        ctx->tm.stage_keys_exchanged[s] = sum;
+    }
 }
 
 // Fill timings after all events completed.
@@ -848,7 +1168,7 @@ int msort_rank_mode(int device) {
         cudaGetLastError();
         return -1;
     }
-    const int r = atomic_rank_ok() ? 1 : 0;
+    const int r = atomic_rank_ok(nullptr) ? 1 : 0;
     cudaSetDevice(prev);
     return r;
 }
@@ -909,7 +1229,7 @@ int msort_step_radix_pass(const void* d_in, void* d_out, uint64_t n, int key_typ
     RadixWs ws = radix_ws_layout(d_ws, n, key_type);
     CUDA_TRY(cudaMemsetAsync(ws.counters, 0, ws.zero_bytes, st));
     CUDA_TRY(launch_scan(d_hist, ws.base, ws.trivial, n, key_type, st));
-    CUDA_TRY(launch_onesweep(d_in, d_out, n, key_type, pass, (flags & 3) | (atomic_rank_ok() ? 4 : 0), ws,
+    CUDA_TRY(launch_onesweep(d_in, d_out, n, key_type, pass, (flags & 3) | (atomic_rank_ok(st) ? 4 : 0), ws,
                              ws.base + pass * 256, st));
     return MSORT_OK;
 }
@@ -926,7 +1246,7 @@ int msort_radix_sort(void* d_keys, void* d_aux, uint64_t n, int key_type, void* 
     for (int p = 0; p < P; ++p) {
         const void* in = (p % 2 == 0) ? d_keys : d_aux;
         void* out = (p % 2 == 0) ? d_aux : d_keys;
-        const int flags = (p == 0 ? 1 : 0) | (p == P - 1 ? 2 : 0) | ((p == 0 || atomic_rank_ok()) ? 4 : 0);
+        const int flags = (p == 0 ? 1 : 0) | (p == P - 1 ? 2 : 0) | ((p == 0 || atomic_rank_ok(st)) ? 4 : 0);
         CUDA_TRY(launch_onesweep(in, out, n, key_type, p, flags, ws, ws.base + p * 256, st));
     }
     return MSORT_OK;
@@ -1013,6 +1333,14 @@ int msort_create(msort_ctx** out, int n_gpus, const int* device_ids, uint64_t ma
             return s;
         }
     }
+    if (n_gpus > 1) {
+        const int s = peer_bulk_selftest_local(ctx.get());
+        if (s == MSORT_OK) apply_exchange_mode(ctx.get());
+        if (s != MSORT_OK) {
+            for (int j = 0; j < n_gpus; ++j) free_rank(ctx->r[j]);
+            return s;
+        }
+    }
     *out = ctx.release();
     return MSORT_OK;
 }
@@ -1025,6 +1353,7 @@ int msort_destroy(msort_ctx* ctx) {
         for (void* p : ctx->opened) cudaIpcCloseMemHandle(p);
         if (ctx->my_flags) cudaFree(ctx->my_flags);
     }
+    nccl_destroy(ctx->nccl);
     for (int i = 0; i < ctx->nlocal; ++i) free_rank(ctx->r[i]);
     delete ctx;
     return MSORT_OK;
@@ -1038,16 +1367,24 @@ int msort_set_option(msort_ctx* ctx, int option, int64_t value) {
         case MSORT_OPT_SKIP_TRIVIAL: ctx->skip_trivial = value ? 1 : 0; return MSORT_OK;
         case MSORT_OPT_HOST_PIPELINE: ctx->host_pipeline = value ? 1 : 0; return MSORT_OK;
         case MSORT_OPT_SMALL_GRAPH: ctx->small_graph = value ? 1 : 0; return MSORT_OK;
+        case MSORT_OPT_STOP_AFTER_STAGE:  // testing: -1 = run every stage
+            ctx->stop_after = value < 0 ? -1 : int(std::min<int64_t>(value, MSORT_MAX_STAGES));
+            return MSORT_OK;
+        case MSORT_OPT_RADIX_EPOCH:  // testing: the next sort runs at epoch value + 1 (mod the tag cycle)
+            if (value < 0 || value >= int64_t(kEpochs)) return set_error(MSORT_ERR_INVALID_ARGUMENT, "epoch 0..511");
+            for (int i = 0; i < ctx->nlocal; ++i) ctx->r[i].radix_epoch = uint32_t(value);
+            return MSORT_OK;
         case MSORT_OPT_EXCHANGE:
-            if (value < 0 || value > 3) return set_error(MSORT_ERR_INVALID_ARGUMENT, "exchange mode 0, 1, 2 or 3");
-            if (value == 1)
+            if (value < 0 || value > 4) return set_error(MSORT_ERR_INVALID_ARGUMENT, "exchange mode 0..4");
+            if (value == 1 || value == 4)  // a receive buffer per rank
                 for (int i = 0; i < ctx->nlocal; ++i)
                     if (!ctx->r[i].buf[2]) {
                         CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
                         CUDA_TRY(cudaMalloc(&ctx->r[i].buf[2], std::max<size_t>(ctx->cap * key_bytes(ctx->kt), 256)));
                     }
+            if (value == 4 && !ctx->dist && ctx->nccl.comms.empty()) MSORT_TRY(nccl_init_local(ctx));
             ctx->exchange = int(value);
-            return MSORT_OK;
+            return apply_exchange_mode(ctx);
         default: return set_error(MSORT_ERR_INVALID_ARGUMENT, "unknown option");
     }
 }
@@ -1108,6 +1445,7 @@ int msort_sort_device(msort_ctx* ctx, void* const* chunks, uint64_t keys_per_gpu
             CUDA_TRY(cudaStreamWaitEvent(static_cast<cudaStream_t>(streams[i]), ctx->r[i].e_end, 0));
         }
     MSORT_TRY(finish_local(ctx));
+    if (ctx->stats_on_device) stage_stats_from_device(ctx, *ctx->r[0].h_stage, keys_per_gpu);
     collect_timings(ctx, ctx->g);
     collect_exchange_timings(ctx);
     ctx->tm.total_ms = ctx->tm.sort_ms + ctx->tm.merge_ms;
@@ -1270,6 +1608,7 @@ int msort_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n) {
         CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
         CUDA_TRY(cudaEventSynchronize(ctx->r[i].e_d2h1));
     }
+    if (ctx->stats_on_device) stage_stats_from_device(ctx, *ctx->r[0].h_stage, c);
     collect_timings(ctx, g);
     collect_exchange_timings(ctx);
     for (int i = 0; i < g; ++i) {
@@ -1412,6 +1751,8 @@ int msort_dist_export(msort_ctx* ctx, void* handle_out) {
     return MSORT_OK;
 }
 
+static int dist_barrier(msort_ctx* ctx);
+
 int msort_dist_import(msort_ctx* ctx, const void* all_handles) {
     if (!ctx || !ctx->dist || !all_handles) return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad argument");
     DeviceGuard guard;
@@ -1440,6 +1781,27 @@ int msort_dist_import(msort_ctx* ctx, const void* all_handles) {
         ctx->peer_flags[q] = static_cast<unsigned long long*>(p);
     }
     ctx->imported = true;
+    // self-test of bulk copies from every peer's mapping (collective: every rank
+    // writes its odd pattern, a device barrier, merges reading each peer, a
+    // barrier before anyone's B0 is reused)
+    if (ctx->g > 1 && ctx->cap >= 2 * uint64_t(kSelfTestKeys)) {
+        Rank& R = ctx->r[0];
+        std::vector<uint32_t> even, odd;
+        selftest_pattern(even, odd, kSelfTestKeys);
+        CUDA_TRY(cudaMemcpy(R.buf[0], odd.data(), kSelfTestKeys * 4, cudaMemcpyHostToDevice));
+        MSORT_TRY(dist_barrier(ctx));
+        for (int q = 0; q < ctx->g; ++q) {
+            if (q == ctx->rank) continue;
+            bool ok = false;
+            const int st = selftest_merge(ctx, R, ctx->peer_buf[q][0], kSelfTestKeys, &ok);
+            if (st != MSORT_OK || !ok) ctx->peer_bulk_ok = false;
+        }
+        MSORT_TRY(dist_barrier(ctx));
+        CUDA_TRY(cudaMemcpyAsync(R.h_err, R.d_err, sizeof(int), cudaMemcpyDeviceToHost, R.st));
+        CUDA_TRY(cudaStreamSynchronize(R.st));
+        if (*R.h_err) return set_error(MSORT_ERR_TIMEOUT, "device barrier timed out during the peer self-test");
+        MSORT_TRY(apply_exchange_mode(ctx));
+    }
     return MSORT_OK;
 }
 
@@ -1460,16 +1822,187 @@ static int dist_barrier(msort_ctx* ctx) {
     return MSORT_OK;
 }
 
+// c = chunk keys, valid = real keys in it (the rest is padded here, reading Q3)
 static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream, bool keep_timings,
-                          const char* host = nullptr);
+                          const char* host, uint64_t valid);
 
-int msort_dist_sort(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream) {
-    return dist_sort_impl(ctx, d_chunk, c, stream, false);
+int msort_plan_chunk(uint64_t n, int g, int rank, uint64_t* c, uint64_t* offset, uint64_t* valid) {
+    if (!valid_g(g) || rank < 0 || rank >= g) return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad g or rank");
+    const uint64_t cc = chunk_size(n, g);
+    const uint64_t lo = std::min<uint64_t>(n, uint64_t(rank) * cc);
+    if (c) *c = cc;
+    if (offset) *offset = lo;
+    if (valid) *valid = std::min<uint64_t>(n - lo, cc);
+    return MSORT_OK;
 }
 
-int msort_dist_sort_host(msort_ctx* ctx, void* host_keys, uint64_t c) {
+// --- interconnect peaks ----------------------------------------------------------
+
+// One timed pattern over the ranks this process drives: `issue(i)` enqueues rank
+// i's copies on its streams; every stream first waits for every rank's start
+// marker (they start together), the time is the slowest rank's.  Dist mode: a
+// device barrier lines the processes up instead.
+}  // extern "C"
+template <class Issue>
+static int time_pattern(msort_ctx* ctx, int reps, Issue issue, double* ms_out) {
+    const int nl = ctx->nlocal;
+    double tot = 0;
+    for (int r = 0; r < reps + 1; ++r) {
+        if (ctx->dist) {
+            Rank& R = ctx->r[0];
+            CUDA_TRY(cudaSetDevice(R.dev));
+            MSORT_TRY(dist_barrier(ctx));
+        }
+        for (int i = 0; i < nl; ++i) {
+            CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
+            CUDA_TRY(cudaEventRecord(ctx->r[i].e_sync[0], ctx->r[i].st));
+        }
+        for (int i = 0; i < nl; ++i) {
+            Rank& R = ctx->r[i];
+            CUDA_TRY(cudaSetDevice(R.dev));
+            for (int q = 0; q < nl; ++q)
+                if (q != i) CUDA_TRY(cudaStreamWaitEvent(R.st, ctx->r[q].e_sync[0], 0));
+            CUDA_TRY(cudaEventRecord(R.e_begin, R.st));
+            CUDA_TRY(cudaStreamWaitEvent(R.cst, R.e_begin, 0));
+            MSORT_TRY(issue(i));
+            CUDA_TRY(cudaEventRecord(R.e_merged, R.cst));
+            CUDA_TRY(cudaStreamWaitEvent(R.st, R.e_merged, 0));
+            CUDA_TRY(cudaEventRecord(R.e_end, R.st));
+        }
+        double mx = 0;
+        for (int i = 0; i < nl; ++i) {
+            Rank& R = ctx->r[i];
+            CUDA_TRY(cudaSetDevice(R.dev));
+            CUDA_TRY(cudaEventSynchronize(R.e_end));
+            mx = std::max(mx, double(elapsed(R.e_begin, R.e_end)));
+        }
+        if (r > 0) tot += mx;
+    }
+    if (ctx->dist && ctx->g > 1) {  // peers are done reading our buffers
+        CUDA_TRY(cudaSetDevice(ctx->r[0].dev));
+        MSORT_TRY(dist_barrier(ctx));
+        CUDA_TRY(cudaStreamSynchronize(ctx->r[0].st));
+    }
+    *ms_out = tot / std::max(1, reps);
+    return MSORT_OK;
+}
+extern "C" {
+
+int msort_measure_links(msort_ctx* ctx, uint64_t bytes, int reps, msort_link_peaks* out) {
+    if (!ctx || !out || reps < 1) return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad argument");
+    if (ctx->dist && !ctx->imported) return set_error(MSORT_ERR_INVALID_ARGUMENT, "dist ctx not imported");
+    DeviceGuard guard;
+    const int g = ctx->g, nl = ctx->nlocal;
+    bytes = std::min<uint64_t>(bytes, ctx->cap * key_bytes(ctx->kt)) / 4096 * 4096;
+    if (bytes == 0) return set_error(MSORT_ERR_INVALID_ARGUMENT, "bytes below one page");
+    *out = msort_link_peaks{};
+    out->bytes = bytes;
+    out->pairs = g / 2;
+    for (int i = 0; i < nl; ++i) {
+        CUDA_TRY(cudaSetDevice(ctx->r[i].dev));
+        CUDA_TRY(cudaDeviceSynchronize());
+    }
+    // mirrored pairs: rank i pulls from rank g-1-i's B0 into its staging chunk, all pairs at once
+    auto src_of = [&](int i) -> const void* {
+        const int me = ctx->dist ? ctx->rank : i, p = g - 1 - me;
+        return ctx->dist ? ctx->peer_buf[p][0] : ctx->r[p].buf[0];
+    };
+    if (g > 1) {
+        int same = 0;
+        if (ctx->dist) {
+            same = -1;  // unknown across processes (the caller knows its device map)
+        } else {
+            for (int i = 0; i < g; ++i) same |= ctx->r[i].dev == ctx->r[g - 1 - i].dev;
+        }
+        out->same_device = same;
+        double ms = 0;
+        MSORT_TRY(time_pattern(ctx, reps, [&](int i) -> int {
+            CUDA_TRY(cudaMemcpyAsync(ctx->r[i].stage, src_of(i), bytes, cudaMemcpyDefault, ctx->r[i].st));
+            return MSORT_OK;
+        }, &ms));
+        out->p2p_ce_gbs = bytes / (ms * 1e6);
+        MSORT_TRY(time_pattern(ctx, reps, [&](int i) -> int {
+            CUDA_TRY(launch_copy_sm(ctx->r[i].stage, src_of(i), bytes, ctx->r[i].st, sm_count_of(ctx->r[i].dev)));
+            return MSORT_OK;
+        }, &ms));
+        out->p2p_sm_gbs = bytes / (ms * 1e6);
+    }
+    // PCIe (§4.2): pinned host buffers per GPU, all GPUs concurrently
+    std::vector<void*> hin(nl, nullptr), hout(nl, nullptr);
+    int st = MSORT_OK;
+    for (int i = 0; i < nl && st == MSORT_OK; ++i) {
+        if (cudaMallocHost(&hin[i], bytes) != cudaSuccess || cudaMallocHost(&hout[i], bytes) != cudaSuccess) {
+            cudaGetLastError();
+            st = set_error(MSORT_ERR_OUT_OF_MEMORY, "pinned host buffers for the PCIe measurement");
+        } else {
+            std::memset(hin[i], 0x5A, bytes);
+        }
+    }
+    double ms = 0;
+    if (st == MSORT_OK)
+        st = time_pattern(ctx, reps, [&](int i) -> int {
+            CUDA_TRY(cudaMemcpyAsync(ctx->r[i].stage, hin[i], bytes, cudaMemcpyHostToDevice, ctx->r[i].st));
+            return MSORT_OK;
+        }, &ms);
+    if (st == MSORT_OK) out->h2d_gbs = bytes / (ms * 1e6);
+    if (st == MSORT_OK)
+        st = time_pattern(ctx, reps, [&](int i) -> int {
+            CUDA_TRY(cudaMemcpyAsync(hout[i], ctx->r[i].buf[0], bytes, cudaMemcpyDeviceToHost, ctx->r[i].st));
+            return MSORT_OK;
+        }, &ms);
+    if (st == MSORT_OK) out->d2h_gbs = bytes / (ms * 1e6);
+    if (st == MSORT_OK)
+        st = time_pattern(ctx, reps, [&](int i) -> int {
+            CUDA_TRY(cudaMemcpyAsync(ctx->r[i].stage, hin[i], bytes, cudaMemcpyHostToDevice, ctx->r[i].st));
+            CUDA_TRY(cudaMemcpyAsync(hout[i], ctx->r[i].buf[0], bytes, cudaMemcpyDeviceToHost, ctx->r[i].cst));
+            return MSORT_OK;
+        }, &ms);
+    if (st == MSORT_OK) out->bidir_gbs = bytes / (ms * 1e6);
+    for (int i = 0; i < nl; ++i) {
+        cudaSetDevice(ctx->r[i].dev);
+        cudaDeviceSynchronize();
+        if (hin[i]) cudaFreeHost(hin[i]);
+        if (hout[i]) cudaFreeHost(hout[i]);
+    }
+    return st;
+}
+
+int msort_nccl_unique_id(void* out) {
+    if (!out) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL out");
+    std::string err;
+    if (!nccl_unique_id(out, &err)) return set_error(MSORT_ERR_NCCL, err);
+    return MSORT_OK;
+}
+
+int msort_dist_nccl_init(msort_ctx* ctx, const void* unique_id) {
+    if (!ctx || !ctx->dist || !unique_id) return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad argument");
+    DeviceGuard guard;
+    CUDA_TRY(cudaSetDevice(ctx->r[0].dev));
+    nccl_destroy(ctx->nccl);
+    std::string err;
+    if (!nccl_init_rank(ctx->nccl, ctx->g, unique_id, ctx->rank, &err)) return set_error(MSORT_ERR_NCCL, err);
+    return MSORT_OK;
+}
+
+int msort_release_cached(void) {
+    std::lock_guard<std::mutex> lock(g_cache_mu);
+    for (auto& kv : g_cache) msort_destroy(kv.second);
+    g_cache.clear();
+    return MSORT_OK;
+}
+
+int msort_dist_sort(msort_ctx* ctx, void* d_chunk, uint64_t n_total, void* stream) {
+    if (!ctx || !ctx->dist) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL or non-dist ctx");
+    uint64_t c = 0, valid = 0;
+    MSORT_TRY(msort_plan_chunk(n_total, ctx->g, ctx->rank, &c, nullptr, &valid));
+    return dist_sort_impl(ctx, d_chunk, c, stream, false, nullptr, valid);
+}
+
+int msort_dist_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n_total) {
     if (!ctx || !ctx->dist || !ctx->imported) return set_error(MSORT_ERR_INVALID_ARGUMENT, "dist ctx not imported");
-    if (c && !host_keys) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL keys");
+    uint64_t c = 0, valid = 0;
+    MSORT_TRY(msort_plan_chunk(n_total, ctx->g, ctx->rank, &c, nullptr, &valid));
+    if (valid && !host_keys) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL keys");
     MSORT_TRY(check_c(ctx, c));
     DeviceGuard guard;
     Rank& R = ctx->r[0];
@@ -1477,16 +2010,16 @@ int msort_dist_sort_host(msort_ctx* ctx, void* host_keys, uint64_t c) {
     reset_timings(ctx, c);
     const size_t K = key_bytes(ctx->kt);
     if (ctx->host_pipeline && c >= kPipeMinKeys) {
-        // pipelined S0 (MSORT_OPT_HOST_PIPELINE): H2D pieces sorted as they land
-        MSORT_TRY(dist_sort_impl(ctx, R.stage, c, R.st, true, static_cast<const char*>(host_keys)));
+        // pipelined S0 (MSORT_OPT_HOST_PIPELINE): H2D pieces sorted as they land (the pad is filled there)
+        MSORT_TRY(dist_sort_impl(ctx, R.stage, c, R.st, true, static_cast<const char*>(host_keys), valid));
     } else {
         CUDA_TRY(cudaEventRecord(R.e_h2d0, R.st));
-        if (c) CUDA_TRY(cudaMemcpyAsync(R.stage, host_keys, c * K, cudaMemcpyHostToDevice, R.st));
+        if (valid) CUDA_TRY(cudaMemcpyAsync(R.stage, host_keys, valid * K, cudaMemcpyHostToDevice, R.st));
         CUDA_TRY(cudaEventRecord(R.e_h2d1, R.st));
-        MSORT_TRY(dist_sort_impl(ctx, R.stage, c, R.st, true));
+        MSORT_TRY(dist_sort_impl(ctx, R.stage, c, R.st, true, nullptr, valid));
     }
     CUDA_TRY(cudaEventRecord(R.e_d2h0, R.st));
-    if (c) CUDA_TRY(cudaMemcpyAsync(host_keys, R.stage, c * K, cudaMemcpyDeviceToHost, R.st));
+    if (valid) CUDA_TRY(cudaMemcpyAsync(host_keys, R.stage, valid * K, cudaMemcpyDeviceToHost, R.st));
     CUDA_TRY(cudaEventRecord(R.e_d2h1, R.st));
     CUDA_TRY(cudaEventSynchronize(R.e_d2h1));
     ctx->tm.h2d_ms = elapsed(R.e_h2d0, R.e_h2d1);
@@ -1496,7 +2029,7 @@ int msort_dist_sort_host(msort_ctx* ctx, void* host_keys, uint64_t c) {
 }
 
 static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream, bool keep_timings,
-                          const char* host) {
+                          const char* host, uint64_t valid) {
     if (!ctx || !ctx->dist || !ctx->imported) return set_error(MSORT_ERR_INVALID_ARGUMENT, "dist ctx not imported");
     if (c && !d_chunk) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL chunk");
     MSORT_TRY(check_c(ctx, c));
@@ -1518,18 +2051,22 @@ static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* strea
     void* sorted_dst = g == 1 ? d_chunk : R.buf[1];
     if (host) {
         uint64_t split = 0;
-        MSORT_TRY(load_sort_pieces(ctx, R, host, c, c, static_cast<char*>(d_chunk), &split));
+        MSORT_TRY(load_sort_pieces(ctx, R, host, valid, c, static_cast<char*>(d_chunk), &split));
         const char* b0 = static_cast<const char*>(R.buf[0]);
         CUDA_TRY(launch_merge(b0, split, b0 + split * key_bytes(ctx->kt), c - split, sorted_dst, ctx->kt, R.mws, R.st,
                               &ctx->tm.kernel_launches));
     } else {
+        if (valid < c) {  // reading Q3: pad with the largest key under T
+            CUDA_TRY(launch_fill_max(static_cast<char*>(d_chunk) + valid * key_bytes(ctx->kt), c - valid, ctx->kt, R.st));
+            ctx->tm.kernel_launches += 1;
+        }
         MSORT_TRY(radix_begin(ctx, R, d_chunk, c));
         if (ctx->skip_trivial) CUDA_TRY(cudaStreamSynchronize(R.st));
         MSORT_TRY(radix_passes(ctx, R, d_chunk, sorted_dst, R.buf[0], c));
     }
     for (int q = 0; q < g; ++q) cur[q] = g == 1 ? -1 : 1;
     CUDA_TRY(cudaEventRecord(R.e_sorted, R.st));
-    if (g > 1 && ctx->exchange >= 2) {
+    if (g > 1 && (ctx->xmode == 2 || ctx->xmode == 3)) {
         // NEXT-1: splitters from every peer's sorted chunk, one pull per peer,
         // barrier (peers' B1 no longer read), local merge tree into d_chunk
         const size_t K = key_bytes(ctx->kt);
@@ -1547,7 +2084,7 @@ static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* strea
         std::vector<uint64_t> s(R.h_pivot, R.h_pivot + (g + 1) * g);
         record_alltoall_stats(ctx, s.data(), g);
         const Runs rr = runs_of(s.data(), g, me);
-        if (ctx->exchange == 2) {
+        if (ctx->xmode == 2) {
             // fused: merge straight out of the peers' B1, then one barrier so that
             // no rank reuses its B1 while a peer may still be reading it
             const char* rp[MSORT_MAX_GPUS];
@@ -1583,46 +2120,86 @@ static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* strea
     std::vector<int> labels;
     stage_labels(g, labels);
     const int S = int(labels.size());
-    ctx->tm.n_stages = S;
-    auto peer_ptr = [&](int q, int which) -> const void* {
-        return which < 0 ? (q == me ? d_chunk : nullptr) : ctx->peer_buf[q][which];
-    };
-    for (int s = 0; s < S; ++s) {
-        const int label = labels[s];
-        const bool last = s == S - 1;
-        MSORT_TRY(dist_barrier(ctx));
-        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[s][0], R.st));
-        GroupPtrs all{};
-        for (int q = 0; q < g; ++q) all.p[q] = peer_ptr(q, cur[q]);
-        const int ngroups = g / label;
-        CUDA_TRY(launch_pivots(all, ngroups, label, c, ctx->kt, R.d_pivot, R.st));
-        ctx->tm.kernel_launches += 1;
-        CUDA_TRY(cudaMemcpyAsync(R.h_pivot, R.d_pivot, ngroups * sizeof(uint64_t), cudaMemcpyDeviceToHost, R.st));
-        CUDA_TRY(cudaMemcpyAsync(R.h_err, R.d_err, sizeof(int), cudaMemcpyDeviceToHost, R.st));
-        CUDA_TRY(cudaStreamSynchronize(R.st));
-        if (*R.h_err) return set_error(MSORT_ERR_TIMEOUT, "device barrier timed out (a peer rank did not arrive)");
-        uint64_t piv[MSORT_MAX_GPUS / 2] = {};
-        for (int j = 0; j < ngroups; ++j) piv[j] = R.h_pivot[j];
-        Exchange ex;
-        plan_exchange(g, label, c, piv, ex);
-        ctx->tm.stage_label[s] = label;
-        uint64_t mx = 0, sum = 0;
-        for (int j = 0; j < ngroups; ++j) ctx->tm.stage_pivot[s][j] = piv[j];
+    const int S_run = stages_to_run(ctx, S);
+    ctx->tm.n_stages = S_run;
+    if (g > 1 && ctx->xmode == 0) {
+        // device-resident Alg.2 (see alg2_device_local): a device barrier per
+        // stage, pivots / exchange / rotation decided on the GPU, no host round trip
+        BufTable bt{};
         for (int q = 0; q < g; ++q) {
-            mx = std::max(mx, ex.x[q]);
-            if (ex.side[q] == 0) sum += ex.x[q];
+            bt.p[q][0] = q == me ? d_chunk : nullptr;  // (peers' user chunks are never read)
+            bt.p[q][1] = ctx->peer_buf[q][0];
+            bt.p[q][2] = ctx->peer_buf[q][1];
         }
-        ctx->tm.stage_max_x[s] = mx;
-        ctx->tm.stage_keys_exchanged[s] = sum;
-        R.cur = cur[me];
-        int mine = cur[me];
-        const void* peer = ex.partner[me] >= 0 ? peer_ptr(ex.partner[me], cur[ex.partner[me]]) : nullptr;
-        MSORT_TRY(launch_exchange(ctx, R, s, last, c, ex.x[me], ex.side[me], peer_ptr(me, cur[me]), peer, mine));
-        if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[s][1], R.st));
-        // replicate every rank's buffer rotation (all ranks see the same pivots)
-        for (int q = 0; q < g; ++q)
-            if (ex.x[q] != 0) cur[q] = last ? -1 : (cur[q] == 0 ? 1 : 0);
-        if (cur[me] != mine) return set_error(MSORT_ERR_INTERNAL, "buffer rotation diverged");
+        CUDA_TRY(launch_stage_init(R.d_stage, g, R.st));
+        ctx->tm.kernel_launches += 1;
+        for (int s = 0; s < S_run; ++s) {
+            MSORT_TRY(dist_barrier(ctx));
+            if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[s][0], R.st));
+            CUDA_TRY(launch_stage_pivots(bt, R.d_stage, s, labels[s], g, c, ctx->kt, R.st));
+            ctx->tm.kernel_launches += 1;
+            if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_xch[s][0], R.st));
+            CUDA_TRY(launch_stage_merge(bt, R.d_stage, R.d_desc, s, labels[s], me, g, c, s == S - 1, ctx->kt, R.mws,
+                                        R.st, &ctx->tm.kernel_launches));
+            if (ctx->timing) {
+                CUDA_TRY(cudaEventRecord(R.e_xch[s][1], R.st));
+                R.xch_rec[s] = true;
+                CUDA_TRY(cudaEventRecord(R.e_stage[s][1], R.st));
+            }
+        }
+        CUDA_TRY(launch_stage_final(bt, R.d_stage, me, c, ctx->kt, R.st, sm_count_of(R.dev)));
+        ctx->tm.kernel_launches += 1;
+        CUDA_TRY(cudaMemcpyAsync(R.h_stage, R.d_stage, sizeof(DevStage), cudaMemcpyDeviceToHost, R.st));
+        ctx->stats_on_device = true;
+        for (int q = 0; q < g; ++q) cur[q] = -1;
+    } else {
+        auto peer_ptr = [&](int q, int which) -> const void* {
+            return which < 0 ? (q == me ? d_chunk : nullptr) : ctx->peer_buf[q][which];
+        };
+        for (int s = 0; s < S_run; ++s) {
+            const int label = labels[s];
+            const bool last = s == S - 1;
+            MSORT_TRY(dist_barrier(ctx));
+            if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[s][0], R.st));
+            GroupPtrs all{};
+            for (int q = 0; q < g; ++q) all.p[q] = peer_ptr(q, cur[q]);
+            const int ngroups = g / label;
+            CUDA_TRY(launch_pivots(all, ngroups, label, c, ctx->kt, R.d_pivot, R.st));
+            ctx->tm.kernel_launches += 1;
+            CUDA_TRY(cudaMemcpyAsync(R.h_pivot, R.d_pivot, ngroups * sizeof(uint64_t), cudaMemcpyDeviceToHost, R.st));
+            CUDA_TRY(cudaMemcpyAsync(R.h_err, R.d_err, sizeof(int), cudaMemcpyDeviceToHost, R.st));
+            CUDA_TRY(cudaStreamSynchronize(R.st));
+            if (*R.h_err) return set_error(MSORT_ERR_TIMEOUT, "device barrier timed out (a peer rank did not arrive)");
+            uint64_t piv[MSORT_MAX_GPUS / 2] = {};
+            for (int j = 0; j < ngroups; ++j) piv[j] = R.h_pivot[j];
+            Exchange ex;
+            plan_exchange(g, label, c, piv, ex);
+            ctx->tm.stage_label[s] = label;
+            uint64_t mx = 0, sum = 0;
+            for (int j = 0; j < ngroups; ++j) ctx->tm.stage_pivot[s][j] = piv[j];
+            for (int q = 0; q < g; ++q) {
+                mx = std::max(mx, ex.x[q]);
+                if (ex.side[q] == 0) sum += ex.x[q];
+            }
+            ctx->tm.stage_max_x[s] = mx;
+            ctx->tm.stage_keys_exchanged[s] = sum;
+            R.cur = cur[me];
+            int mine = cur[me];
+            if (ctx->xmode == 4) {
+                if (ctx->nccl.comms.empty())
+                    return set_error(MSORT_ERR_NCCL, "exchange mode 4 needs msort_dist_nccl_init first");
+                if (ctx->timing && ex.x[me]) CUDA_TRY(cudaEventRecord(R.e_xch[s][0], R.st));
+                R.user = d_chunk;
+                MSORT_TRY(nccl_stage_exchange(ctx, ex, c, last));
+            }
+            const void* peer = ex.partner[me] >= 0 ? peer_ptr(ex.partner[me], cur[ex.partner[me]]) : nullptr;
+            MSORT_TRY(launch_exchange(ctx, R, s, last, c, ex.x[me], ex.side[me], peer_ptr(me, cur[me]), peer, mine));
+            if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_stage[s][1], R.st));
+            // replicate every rank's buffer rotation (all ranks see the same pivots)
+            for (int q = 0; q < g; ++q)
+                if (ex.x[q] != 0) cur[q] = last ? -1 : (cur[q] == 0 ? 1 : 0);
+            if (cur[me] != mine) return set_error(MSORT_ERR_INTERNAL, "buffer rotation diverged");
+        }
     }
     if (cur[me] != -1)
         CUDA_TRY(cudaMemcpyAsync(d_chunk, ctx->peer_buf[me][cur[me]], c * key_bytes(ctx->kt), cudaMemcpyDeviceToDevice, R.st));
@@ -1632,6 +2209,7 @@ static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* strea
     CUDA_TRY(cudaStreamWaitEvent(ust, R.e_end, 0));
     CUDA_TRY(cudaStreamSynchronize(R.st));
     if (*R.h_err) return set_error(MSORT_ERR_TIMEOUT, "device barrier timed out (a peer rank did not arrive)");
+    if (ctx->stats_on_device) stage_stats_from_device(ctx, *R.h_stage, c);
     collect_timings(ctx, 1);
     collect_exchange_timings(ctx);
     ctx->tm.total_ms = ctx->tm.sort_ms + ctx->tm.merge_ms;

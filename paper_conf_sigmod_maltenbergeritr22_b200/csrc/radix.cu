@@ -12,9 +12,9 @@
 //   onesweep_kernel  persistent blocks; per tile: block digit counts, stable
 //                    warp ranking (lane-ordered smem atomics, or atomicOr /
 //                    8-ballot peer masks), decoupled look-back across tiles
-//                    (windowed, with per-group aggregates) for the global
-//                    digit offset, smem staging, coalesced scatter (S3); the
-//                    next tile's keys load during the scatter
+//                    (32-bit group-relative status words, per-group bases)
+//                    for the global digit offset, smem staging, coalesced
+//                    scatter (S3); the next tile's keys load during the scatter
 // The float codec T (reading Q1) is applied on the first pass's load and T^-1
 // on the last pass's store (S1), so no separate codec pass touches HBM.
 #include <atomic>
@@ -155,11 +155,22 @@ __global__ void __launch_bounds__(kRadix) scan_kernel(const uint32_t* __restrict
 // keys/cycle/SM, while shared memory serves 1 wavefront (128 B)/cycle/SM and
 // the integer ALU pipe 2 warp-instructions/cycle/SM; a random 4-byte smem
 // access by 32 lanes costs ~3.5 wavefronts (bank conflicts) and MATCH.ANY
-// ~60 ADU cycles.  The ranking therefore mixes two peer-mask methods per item
-// (compile-time pattern): an 8-ballot match (ALU only) and an smem atomicOr
-// mask (3 smem ops), so both pipes work in parallel.  Per-warp digit counts are
-// taken first ("early counts"), the tile aggregate is published before the
-// ranking, and the ranking's leader atomicAdd returns the final smem slot.
+// ~60 ADU cycles.  Per tile: per-warp digit counts first ("early counts"), the
+// tile aggregate is published before the ranking, and the ranking's atomic
+// returns the key's final smem slot (lane-ordered shared atomics, or a peer
+// match that mixes an 8-ballot match (ALU) with an smem atomicOr mask).
+//
+// Decoupled look-back: one 64-bit status word per (tile, digit),
+//   flag << 62 | tag << 32 | count       (tag = epoch << 4 | pass + 1)
+//   AGG  count = the tile's count of digit d;  INCL  count = inclusive count
+//   over all tiles up to this one.  A tile walks its predecessors inside its
+//   GROUP of kGroup tiles (kLookback words per round), then whole earlier
+//   groups through the last tile's INCL word or the group aggregate
+//   gagg[grp][d] = tiles << 32 | sum (complete when tiles == kGroup).
+// (Round 2 measured a 32-bit variant with group-relative counts and
+// per-group published bases: u32 no faster, u64 7% slower - every tile then
+// needs the group base, one more dependent L2 round trip; not adopted,
+// profiles/radix_tuning_r2.md.)
 // ---------------------------------------------------------------------------
 constexpr unsigned long long kFlagAgg = 1ull, kFlagIncl = 2ull;
 
@@ -167,7 +178,10 @@ __device__ __forceinline__ unsigned long long pack_status(unsigned long long fla
     return (flag << 62) | (uint64_t(tag & 0x3FFFFFFFu) << 32) | count;
 }
 
-// Lanes of the warp whose 8-bit digit equals this lane's (8 ballots).
+// Lanes of the warp whose 8-bit digit equals this lane's (8 ballots).  The
+// and / setp / vote.ballot / conditional-not sequence per bit is the standard
+// 8-ballot peer-match idiom (CUB's warp_matcher_t::match_any in cub/util_ptx.cuh
+// uses the same one).
 __device__ __forceinline__ uint32_t ballot_match8(uint32_t d) {
     uint32_t peers = 0xffffffffu;
 #pragma unroll
@@ -184,26 +198,23 @@ __device__ __forceinline__ uint32_t ballot_match8(uint32_t d) {
     return peers;
 }
 
-// THREADS x ITEMS keys per tile; bit i of BALLOT_MASK: item i ranks with the
-// ballot match (else smem atomicOr); MINB blocks per SM for __launch_bounds__.
-template <int THREADS_, int ITEMS_, uint32_t BALLOT_MASK_, int MINB_, bool PF_, int LB_ = 4, bool ELB_ = false,
-          bool CR_ = false, int GROUP_ = 8, bool CE_ = false>
+// THREADS x ITEMS keys per tile; bit i of BALLOT_MASK: item i of the peer-match
+// ranking uses the ballot match (else smem atomicOr); MINB blocks per SM;
+// LB = look-back window (status loads per round); GROUP = look-back group
+// (tiles); CE = count the prefetched next tile right after this tile's scatter
+// (per-warp counter zeroing, no end-of-tile barrier).
+template <int THREADS_, int ITEMS_, uint32_t BALLOT_MASK_, int MINB_, int LB_, int GROUP_, bool CE_>
 struct OsCfg {
-    // prefetch configs: count the next tile's keys right after this tile's scatter
-    // (per-warp zeroing, no end-of-tile barrier), so a claimed tile publishes its
-    // aggregate sooner
-    static constexpr bool kCountEnd = CE_;
-    static constexpr uint32_t kGroup = GROUP_;  // look-back group size (tiles); 0 = tile-by-tile walk only
-    static constexpr bool kCountRank = CR_;  // atomic-ranked passes: rank = the count atomic's return
-    static constexpr bool kEarlyLookback = ELB_;  // look back right after publishing (before the ranking)
-    static constexpr bool kPrefetch = PF_;  // load the next tile's keys into registers during the scatter
-    static constexpr int kLookback = LB_;  // look-back window (independent status loads per round)
     static constexpr int kThreads = THREADS_;
     static constexpr int kItems = ITEMS_;
     static constexpr uint32_t kBallotMask = BALLOT_MASK_;
     static constexpr int kMinBlocks = MINB_;
+    static constexpr int kLookback = LB_;
+    static constexpr uint32_t kGroup = GROUP_;
+    static constexpr bool kCountEnd = CE_;
     static constexpr int kWarps = THREADS_ / 32;
     static constexpr uint32_t kTile = uint32_t(THREADS_) * ITEMS_;
+    static_assert(GROUP_ >= 2, "look-back groups");
     static constexpr bool kAnyOr = (BALLOT_MASK_ & ((ITEMS_ >= 32 ? 0u : (1u << ITEMS_)) - 1u)) !=
                                    ((ITEMS_ >= 32 ? 0u : (1u << ITEMS_)) - 1u);
     // (the atomicOr peer masks exist only in the peer-match ranking, STABLE)
@@ -213,6 +224,39 @@ struct OsCfg {
     }
 };
 
+// Product tile configurations (profiles/radix_tuning_r1.md; a tuning build
+// may override single parameters with -DMSORT_W32=4 etc.):
+//   u32/f32: 7168-key tiles, 4 blocks of 256 threads per SM, look-back window 2,
+//            groups of 32, next tile counted after the scatter (3 barriers)
+//   u64/f64: 3584-key tiles, 4 blocks per SM, window 4, groups of 16
+#ifndef MSORT_T32
+#define MSORT_T32 256
+#endif
+#ifndef MSORT_I32
+#define MSORT_I32 28
+#endif
+#ifndef MSORT_B32
+#define MSORT_B32 4
+#endif
+#ifndef MSORT_W32
+#define MSORT_W32 2
+#endif
+#ifndef MSORT_G32
+#define MSORT_G32 32
+#endif
+#ifndef MSORT_W64
+#define MSORT_W64 4
+#endif
+#ifndef MSORT_G64
+#define MSORT_G64 16
+#endif
+#define MSORT_CFG32 OsCfg<MSORT_T32, MSORT_I32, 0x5555555u, MSORT_B32, MSORT_W32, MSORT_G32, true>
+#define MSORT_CFG64 OsCfg<256, 14, 0x1555u, 4, MSORT_W64, MSORT_G64, false>
+using Cfg32 = MSORT_CFG32;
+using Cfg64 = MSORT_CFG64;
+template <typename U>
+using CfgOf = std::conditional_t<sizeof(U) == 4, Cfg32, Cfg64>;
+
 // STABLE = false: "atomic ranking": each key takes its smem slot with ONE
 // shared-memory atomicAdd on its warp's digit counter (no peer match).  The
 // order in which lanes of one warp instruction that hit the same counter
@@ -221,12 +265,6 @@ struct OsCfg {
 // ranking stable.  atomic_rank_ok() verifies this on the running GPU once per
 // device (rank_probe_kernel) before any stable pass uses it; the first LSD pass
 // may use it regardless (nothing has ordered the keys yet).
-#ifndef MSORT_ABLATE
-#define MSORT_ABLATE 0  // timing ablations (tools/ablate_build.py); never set in a real build
-#endif
-#if MSORT_ABLATE & 8
-__device__ unsigned long long g_lb_stats[4];  // tiles, window rounds, polls, status loads
-#endif
 template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg, bool STABLE = true>
 __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     onesweep_kernel(const U* __restrict__ in, U* __restrict__ out, uint32_t n, uint32_t shift,
@@ -237,8 +275,9 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     constexpr int ITEMS = Cfg::kItems;
     constexpr int WARPS = Cfg::kWarps;
     constexpr uint32_t TILE = Cfg::kTile;
+    constexpr uint32_t G = Cfg::kGroup;
+    constexpr int W = Cfg::kLookback;
     static_assert(THREADS >= kRadix, "one thread per digit in the look-back");
-    static_assert((TILE * sizeof(U)) % 16 == 0, "bulk copies move whole 16-byte units");
 
     extern __shared__ __align__(128) unsigned char smem_raw[];
     U* s_keys = reinterpret_cast<U*>(smem_raw);                           // digit-ordered staging
@@ -252,6 +291,9 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     const uint32_t ntiles = uint32_t((uint64_t(n) + TILE - 1) / TILE);  // (64-bit: n may be 2^32 - 4)
     const uint32_t lt = lanemask_lt();
     const uint32_t wofs = uint32_t(warp) * 32 * ITEMS + lane;
+    // high word of a status entry: flag << 30 | tag
+    const uint32_t hi_agg = uint32_t(kFlagAgg << 30) | (tag & 0x3FFFFFFFu);
+    const uint32_t hi_incl = uint32_t(kFlagIncl << 30) | (tag & 0x3FFFFFFFu);
 
     // keys of tile t -> registers (warp-striped: warp w owns keys [w*32*ITEMS, (w+1)*32*ITEMS)).
     // Full tiles load raw (encoded by the caller); the partial last tile is
@@ -276,28 +318,17 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     };
 
     // --- decoupled look-back: exclusive count of digit d over all earlier tiles.
-    // Status word per (tile, digit): flag << 62 | tag << 32 | count.  Phase 1
-    // walks the predecessors inside this tile's group of kGroup tiles, a window
-    // of kLookback status words per round (an unpublished predecessor is then
-    // polled alone).  Phase 2 walks whole earlier groups: a group contributes
-    // the inclusive count of its last tile if that is published, else its
-    // aggregate word (tiles << 32 | sum, complete when tiles == kGroup; every
-    // tile adds itself right after counting), so a walk of ~30 tiles takes ~3
-    // rounds instead of ~8.  Publishes this tile's inclusive count.
+    // Phase 1 walks the predecessors inside this tile's group, W status words
+    // per round (an unpublished predecessor is then polled alone).  Phase 2
+    // walks whole earlier groups: a group contributes the inclusive count of
+    // its last tile if that is published, else its aggregate word (complete
+    // when tiles == G; every tile adds itself right after counting), so a walk
+    // of ~30 tiles takes ~3 rounds instead of ~8.  Publishes this tile's
+    // inclusive count.
     auto lookback = [&](const int d, const uint32_t tile, const uint32_t my_total) -> uint32_t {
         uint32_t excl = 0;
-#if MSORT_ABLATE & 1  // timing ablation: no look-back, uniform-share offsets instead
-        excl = uint32_t(uint64_t(tile) * (n >> 8) / ntiles);
-        if (false) {
-#else
         if (tile > 0) {
-#endif
-            // high word of a status entry: flag << 30 | tag
-            const uint32_t hi_agg = uint32_t(kFlagAgg << 30) | (tag & 0x3FFFFFFFu);
-            const uint32_t hi_incl = uint32_t(kFlagIncl << 30) | (tag & 0x3FFFFFFFu);
-            constexpr int W = Cfg::kLookback;
-            constexpr uint32_t G = Cfg::kGroup;
-            const uint32_t first = G ? tile / (G ? G : 1) * G : 0u;  // phase 1 covers tiles [first, tile)
+            const uint32_t first = tile / G * G;  // phase 1 covers tiles [first, tile)
             uint32_t left = tile - first;
             const unsigned long long* p = status + uint64_t(tile - 1) * kRadix + d;
             bool done = false;
@@ -323,25 +354,19 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
                         }
                     }
                 }
-#if MSORT_ABLATE & 8
-                atomicAdd(&g_lb_stats[1], 1ull);
-#endif
                 if (done) break;
-                left -= used;  // (tile 0 is always inclusive, so G == 0 ends above)
+                left -= used;  // (tile 0 is always inclusive)
                 p -= used * kRadix;
                 if (used == 0) {
                     unsigned long long w;
                     do {
                         __nanosleep(32);
-#if MSORT_ABLATE & 8
-                        atomicAdd(&g_lb_stats[2], 1ull);
-#endif
                         w = ld_relaxed_gpu(p);
                     } while (uint32_t(w >> 32) != hi_agg && uint32_t(w >> 32) != hi_incl);
                 }
             }
-            if (G && !done) {
-                uint32_t h = first / (G ? G : 1) - 1;  // newest earlier group not consumed (groups 0..h remain)
+            if (!done) {
+                uint32_t h = first / G - 1;  // newest earlier group not consumed (groups 0..h remain)
                 for (;;) {
                     uint32_t val[W];
                     bool ok[W], inc[W];
@@ -371,23 +396,12 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
                             }
                         }
                     }
-#if MSORT_ABLATE & 8
-                    atomicAdd(&g_lb_stats[1], 1ull);
-#endif
                     if (done || used == h + 1) break;  // (all groups down to 0 consumed)
                     h -= used;
-                    if (used == 0) {
-#if MSORT_ABLATE & 8
-                        atomicAdd(&g_lb_stats[2], 1ull);
-#endif
-                        __nanosleep(32);
-                    }
+                    if (used == 0) __nanosleep(32);
                 }
             }
             st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(kFlagIncl, tag, excl + my_total));
-#if MSORT_ABLATE & 8
-            atomicAdd(&g_lb_stats[0], 1ull);
-#endif
         }
         return excl;
     };
@@ -395,8 +409,8 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     if (Cfg::kAnyOr && STABLE) {  // (atomic-ranked kernels have no peer-mask array)
         for (int i = tid; i < WARPS * kRadix; i += THREADS) (&s_match[0][0])[i] = 0;
     }
-    // per-warp digit counters start at zero; each tile re-zeroes them during its
-    // scatter (they are dead after the ranking), so no barrier of its own
+    // per-warp digit counters start at zero; each tile re-zeroes them during or
+    // after its scatter (they are dead after the ranking)
     auto zero_counts = [&]() {
         uint4* z = reinterpret_cast<uint4*>(&s_cnt[0][0]);
         for (int i = tid; i < WARPS * kRadix / 4; i += THREADS) z[i] = make_uint4(0, 0, 0, 0);
@@ -409,9 +423,8 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
     }
     __syncthreads();
     uint32_t tile = s_next;
-    if (Cfg::kPrefetch && tile < ntiles) load_tile(tile);
-    constexpr bool kCountRank = Cfg::kCountRank && !STABLE;
-    constexpr bool kCE = Cfg::kCountEnd && Cfg::kPrefetch && !kCountRank;
+    if (tile < ntiles) load_tile(tile);
+    constexpr bool kCE = Cfg::kCountEnd;
     auto count_keys = [&]() {
 #pragma unroll
         for (int i = 0; i < ITEMS; ++i) atomicAdd(&s_cnt[warp][uint32_t(keys[i] >> shift) & 0xFF], 1u);
@@ -422,40 +435,16 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
         if (tile >= ntiles) break;
         const uint64_t tile_base = uint64_t(tile) * TILE;
         const bool full = tile_base + TILE <= n;
-        if (!Cfg::kPrefetch) load_tile(tile);
         if (ENC_IN && full && !counted) {
 #pragma unroll
             for (int i = 0; i < ITEMS; ++i) keys[i] = encode<U, FLOAT>(keys[i]);
         }
-        // (s_cnt was zeroed during the previous tile's scatter, or before the loop)
-
-        // --- early counts: per-warp digit histogram (fire-and-forget smem adds).
-        // kCountRank (atomic-ranked passes): the count's returned value is the
-        // key's stable rank within (warp, digit) - lane order, see STABLE - kept
-        // as 16-bit halves, so the ranking below is a plain load, not an atomic.
-        uint32_t rk[kCountRank ? (ITEMS + 1) / 2 : 1];
-        if (kCE && counted) {
-            // counted at the end of the previous tile
-        } else if constexpr (kCountRank) {
-#pragma unroll
-            for (int i = 0; i < ITEMS; ++i) {
-                const uint32_t r = atomicAdd(&s_cnt[warp][uint32_t(keys[i] >> shift) & 0xFF], 1u);
-                if (i & 1) rk[i >> 1] |= r << 16;
-                else rk[i >> 1] = r;
-            }
-        } else
-#pragma unroll
-        for (int i = 0; i < ITEMS; ++i) {
-#if MSORT_ABLATE & 2  // timing ablation only (wrong results): no early counts
-            if (keys[i] == U(0x12345)) 
-#endif
-            atomicAdd(&s_cnt[warp][uint32_t(keys[i] >> shift) & 0xFF], 1u);
-        }
+        // --- early counts: per-warp digit histogram (fire-and-forget smem adds)
+        if (!(kCE && counted)) count_keys();
         __syncthreads();
 
         // --- tile totals -> publish aggregate; per-(warp, digit) smem slot bases
         uint32_t my_total = 0, my_start = 0;
-        uint32_t excl_early = 0;
         uint32_t col[WARPS];  // this digit's per-warp counts (kept for the slot bases)
         if (tid < kRadix) {
             const int d = tid;
@@ -467,8 +456,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
             }
             my_total = sum;
             st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(tile == 0 ? kFlagIncl : kFlagAgg, tag, sum));
-            if constexpr (Cfg::kGroup != 0) atomicAdd(&gagg[uint64_t(tile / Cfg::kGroup) * kRadix + d], (1ull << 32) | sum);
-            if (Cfg::kEarlyLookback) excl_early = lookback(d, tile, sum);
+            atomicAdd(&gagg[uint64_t(tile / G) * kRadix + d], (1ull << 32) | sum);
             uint32_t x = sum;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
@@ -498,10 +486,6 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
 #pragma unroll
         for (int i = 0; i < ITEMS; ++i) {
             const uint32_t d = uint32_t(keys[i] >> shift) & 0xFF;
-            if constexpr (kCountRank) {
-                s_keys[s_cnt[warp][d] + ((rk[i >> 1] >> (16 * (i & 1))) & 0xFFFFu)] = keys[i];
-                continue;
-            }
             if constexpr (!STABLE) {
                 if (hot_on) {
                     // skewed pass: the lanes on one of the 4 most frequent digits
@@ -545,27 +529,19 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
             s_keys[slot] = keys[i];
         }
 
-        // --- look-back (deferred until after the ranking unless kEarlyLookback)
+        // --- look-back (after the ranking: its latency overlaps the other
+        // warps' ranking), then claim the next tile so that its loads can be
+        // issued before (and overlap) this tile's scatter
         if (tid < kRadix) {
             const int d = tid;
-            const uint32_t excl = Cfg::kEarlyLookback ? excl_early : lookback(d, tile, my_total);
+            const uint32_t excl = lookback(d, tile, my_total);
             s_delta[d] = base[d] + excl - my_start;
-            // Prefetch configs claim the next tile here so that its loads can
-            // be issued before (and overlap) this tile's scatter.
-            if (Cfg::kPrefetch && tid == 0) s_next = atomicAdd(tile_counter, 1u);
+            if (tid == 0) s_next = atomicAdd(tile_counter, 1u);
         }
         __syncthreads();
-        if (!Cfg::kPrefetch && tid == 0) {
-            // Claim the next tile only now: a tile id claimed earlier would sit
-            // queued behind this tile while its successors wait for its aggregate.
-            s_next = atomicAdd(tile_counter, 1u);
-        }
-        uint32_t next_tile = 0;
-        if (Cfg::kPrefetch) {
-            // keys[] is dead until the next iteration: its loads fly during the scatter
-            next_tile = s_next;
-            if (next_tile < ntiles) load_tile(next_tile);
-        }
+        // keys[] is dead until the next iteration: its loads fly during the scatter
+        const uint32_t next_tile = s_next;
+        if (next_tile < ntiles) load_tile(next_tile);
 
         // --- scatter: consecutive smem slots of one digit go to consecutive output slots
         if (full) {
@@ -573,17 +549,13 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
             for (int i = 0; i < ITEMS; ++i) {
                 const uint32_t j = tid + i * THREADS;
                 const U k = s_keys[j];
-                uint32_t dst = s_delta[uint32_t(k >> shift) & 0xFF] + j;
-                if (MSORT_ABLATE) dst = min(dst, n - 1);
-                __stcs(out + dst, DEC_OUT ? decode<U, FLOAT>(k) : k);
+                __stcs(out + s_delta[uint32_t(k >> shift) & 0xFF] + j, DEC_OUT ? decode<U, FLOAT>(k) : k);
             }
         } else {
             const uint32_t valid = uint32_t(n - tile_base);
             for (uint32_t j = tid; j < valid; j += THREADS) {
                 const U k = s_keys[j];
-                uint32_t dst = s_delta[uint32_t(k >> shift) & 0xFF] + j;
-                if (MSORT_ABLATE) dst = min(dst, n - 1);
-                out[dst] = DEC_OUT ? decode<U, FLOAT>(k) : k;
+                out[s_delta[uint32_t(k >> shift) & 0xFF] + j] = DEC_OUT ? decode<U, FLOAT>(k) : k;
             }
         }
         if constexpr (kCE) {
@@ -602,80 +574,17 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
                 }
                 count_keys();
             }
-            tile = next_tile;
-            continue;
+        } else {
+            zero_counts();  // for the next tile (ordered before its count atomics by the barrier below)
+            __syncthreads();
         }
-        zero_counts();  // for the next tile (ordered before its count atomics by the barrier below)
-        __syncthreads();
-        tile = Cfg::kPrefetch ? next_tile : s_next;
+        tile = next_tile;
     }
-}
-// Tile configurations (selectable with MSORT_OS_CFG for tuning; 0 = default).
-// OsCfg<threads, keys/thread, ballot mask, blocks/SM, prefetch, look-back
-// window, look-back before ranking, count-rank, look-back group, count at end>; measured on
-// B200 in profiles/radix_tuning_r1.md: config 0 is the fastest for both key
-// widths; the others stay selectable for tuning.
-using Cfg32_0 = OsCfg<256, 28, 0x5555555u, 4, true, 2, false, false, 32, true>;  // 7168-key tiles, 4 blocks of 256,
-                                            // prefetch, look-back window 2, groups of 32, next tile counted after
-                                            // the scatter (best: +0.7% u32, +1.5% f32, +2% zipf vs config 10)
-using Cfg32_1 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 0>;   // tile-by-tile look-back only
-using Cfg32_2 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 16>;  // look-back groups of 16
-using Cfg32_3 = OsCfg<256, 28, 0x5555555u, 4, true, 2, false, false, 64>;  // window 2, look-back groups of 64
-using Cfg32_4 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 32>;  // look-back groups of 32
-using Cfg32_5 = OsCfg<256, 28, 0x5555555u, 4, true, 6, false, false, 32>;  // window 6, groups of 32
-using Cfg32_6 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, true>;       // count atomic's return = rank
-using Cfg32_7 = OsCfg<256, 28, 0x5555555u, 4, true, 1, false, false, 32>;  // window 1, groups of 32
-using Cfg32_8 = OsCfg<256, 24, 0x555555u, 5, true, 2, false, false, 32>;   // 6144-key tiles, 5 blocks/SM (40 warps)
-using Cfg32_9 = OsCfg<256, 20, 0x55555u, 6, true, 2, false, false, 32>;    // 5120-key tiles, 6 blocks/SM (48 warps)
-using Cfg32_10 = OsCfg<256, 28, 0x5555555u, 4, true, 2, false, false, 32>;  // config 0 with the count at the tile's start (4 barriers)
-using Cfg32_11 = OsCfg<256, 28, 0x5555555u, 4, true, 4, false, false, 32, true>;  // config 0 with look-back window 4
-using Cfg32_12 = OsCfg<256, 28, 0x5555555u, 4, true, 2, false, false, 16, true>;  // config 0 with look-back groups of 16
-using Cfg64_0 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 16>;     // prefetch, groups of 16 (best)
-using Cfg64_1 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 0>;      // tile-by-tile look-back only
-using Cfg64_2 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 8>;      // groups of 8
-using Cfg64_3 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 32>;     // groups of 32
-using Cfg64_4 = OsCfg<256, 14, 0x1555u, 4, true, 4, false, false, 16, true>;  // config 0 + next tile counted after the scatter (-3%)
-
-constexpr uint32_t kMinTile32 = 256 * 20;  // smallest u32 tile above (sizes the status array)
-constexpr uint32_t kMinTile64 = 256 * 14;  // smallest u64 tile above
-
-int env_cfg() {
-    static int v = -1;
-    if (v < 0) {
-        const char* e = std::getenv("MSORT_OS_CFG");
-        v = e ? std::atoi(e) : 0;
-        if (v < 0 || v > 12) v = 0;
-    }
-    return v;
 }
 
 __global__ void rank_probe_kernel(uint32_t seed, uint32_t* bad);
 
 std::atomic<int> g_rank_ok[64];  // per device: 0 unknown, 1 lane-ordered, -1 not
-
-bool atomic_rank_ok_impl() {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    if (dev < 0 || dev >= 64) return false;
-    int v = g_rank_ok[dev].load();
-    if (v != 0) return v > 0;
-    const char* e = std::getenv("MSORT_ATOMIC_RANK");
-    if (e && e[0] == '0') {
-        g_rank_ok[dev] = -1;
-        return false;
-    }
-    uint32_t* bad = nullptr;
-    bool ok = false;
-    if (cudaMalloc(&bad, 4) == cudaSuccess && cudaMemset(bad, 0, 4) == cudaSuccess) {
-        rank_probe_kernel<<<592, 256>>>(0x2545F491u, bad);
-        uint32_t hb = 1;
-        if (cudaMemcpy(&hb, bad, 4, cudaMemcpyDeviceToHost) == cudaSuccess) ok = hb == 0;
-    }
-    if (bad) cudaFree(bad);
-    cudaGetLastError();
-    g_rank_ok[dev] = ok ? 1 : -1;
-    return ok;
-}
 
 int sm_count() {
     int dev = 0, count = 0;
@@ -708,9 +617,52 @@ __global__ void __launch_bounds__(256) rank_probe_kernel(uint32_t seed, uint32_t
     }
 }
 
-template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, class Cfg, bool STABLE>
-cudaError_t launch_onesweep_c(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
+// The probe runs once per device on a private stream, outside any capture:
+// called while the caller's stream (or this thread) is capturing a CUDA graph
+// it answers "no" for this call only (the conservative peer-match ranking) and
+// probes later; a failing CUDA call is not cached either, only a measured
+// lane-order mismatch is.
+bool atomic_rank_ok_impl(cudaStream_t caller) {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) {
+        cudaGetLastError();
+        return false;
+    }
+    int v = g_rank_ok[dev].load();
+    if (v != 0) return v > 0;
+    const char* e = std::getenv("MSORT_ATOMIC_RANK");
+    if (e && e[0] == '0') {
+        g_rank_ok[dev] = -1;
+        return false;
+    }
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (caller && cudaStreamIsCapturing(caller, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone) return false;
+    if (cudaStreamIsCapturing(cudaStreamLegacy, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) {
+        cudaGetLastError();  // (a global-mode capture elsewhere forbids the probe's allocations now)
+        return false;
+    }
+    uint32_t* bad = nullptr;
+    cudaStream_t ps = nullptr;
+    int verdict = 0;  // 0: could not run (not cached)
+    if (cudaStreamCreateWithFlags(&ps, cudaStreamNonBlocking) == cudaSuccess && cudaMalloc(&bad, 4) == cudaSuccess &&
+        cudaMemsetAsync(bad, 0, 4, ps) == cudaSuccess) {
+        rank_probe_kernel<<<592, 256, 0, ps>>>(0x2545F491u, bad);
+        uint32_t hb = 1;
+        if (cudaGetLastError() == cudaSuccess && cudaMemcpyAsync(&hb, bad, 4, cudaMemcpyDeviceToHost, ps) == cudaSuccess &&
+            cudaStreamSynchronize(ps) == cudaSuccess)
+            verdict = hb == 0 ? 1 : -1;
+    }
+    if (bad) cudaFree(bad);
+    if (ps) cudaStreamDestroy(ps);
+    cudaGetLastError();
+    if (verdict != 0) g_rank_ok[dev] = verdict;
+    return verdict > 0;
+}
+
+template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, bool STABLE>
+cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
                               const uint32_t* base_row, uint32_t tag, cudaStream_t st, uint32_t hot, bool hot_on) {
+    using Cfg = CfgOf<U>;
     const size_t smem = Cfg::template smem_bytes<U, STABLE>();
     auto kern = onesweep_kernel<U, FLOAT, ENC_IN, DEC_OUT, Cfg, STABLE>;
     // per-device attribute: set on every launch (cheap, and correct when one
@@ -724,44 +676,11 @@ cudaError_t launch_onesweep_c(const void* in, void* out, uint64_t n, int pass, c
     const uint64_t tiles = (n + Cfg::kTile - 1) / Cfg::kTile;
     uint64_t grid = uint64_t(per_sm) * sm_count();
     if (grid > tiles) grid = tiles;
+    const size_t gofs = size_t(pass) * ws.groups * kRadix;
     kern<<<unsigned(grid), Cfg::kThreads, smem, st>>>(reinterpret_cast<const U*>(in), reinterpret_cast<U*>(out),
                                                      uint32_t(n), uint32_t(8 * pass), base_row, ws.status,
-                                                     ws.counters + pass, tag, ws.gagg + size_t(pass) * ws.groups * kRadix,
-                                                     hot, hot_on);
+                                                     ws.counters + pass, tag, ws.gagg + gofs, hot, hot_on);
     return cudaGetLastError();
-}
-
-template <typename U, bool FLOAT, bool ENC_IN, bool DEC_OUT, bool STABLE>
-cudaError_t launch_onesweep_t(const void* in, void* out, uint64_t n, int pass, const RadixWs& ws,
-                              const uint32_t* base_row, uint32_t tag, cudaStream_t st, uint32_t hot, bool hot_on) {
-    const int c = env_cfg();
-    if constexpr (sizeof(U) == 4) {
-        switch (c) {
-            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_1, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_2, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_3, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 4: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_4, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 5: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_5, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 6: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_6, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 7: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_7, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 8: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_8, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 9: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_9, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 10: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_10, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 11: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_11, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 12: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_12, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg32_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-        }
-    } else {
-        switch (c) {
-            case 1: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_1, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 2: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_2, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 3: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_3, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 4: case 10: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_4, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            case 5: case 6: case 7: case 8: case 9:
-                return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-            default: return launch_onesweep_c<U, FLOAT, ENC_IN, DEC_OUT, Cfg64_0, STABLE>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-        }
-    }
 }
 
 template <typename U>
@@ -782,7 +701,7 @@ cudaError_t launch_onesweep_float(const void* in, void* out, uint64_t n, int pas
     if (dec && !enc && atom) return launch_onesweep_t<U, true, false, true, false>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
     if (!enc && !dec && atom) return launch_onesweep_t<U, true, false, false, false>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
     if (enc && dec) return launch_onesweep_t<U, true, true, true, true>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
-    if (enc && (flags & 4)) return launch_onesweep_t<U, true, true, false, false>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
+    if (enc && atom) return launch_onesweep_t<U, true, true, false, false>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
     if (enc) return launch_onesweep_t<U, true, true, false, true>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
     if (dec) return launch_onesweep_t<U, true, false, true, true>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
     return launch_onesweep_t<U, true, false, false, true>(in, out, n, pass, ws, base_row, tag, st, hot, hot_on);
@@ -790,49 +709,22 @@ cudaError_t launch_onesweep_float(const void* in, void* out, uint64_t n, int pas
 
 }  // namespace
 
-bool atomic_rank_ok() { return atomic_rank_ok_impl(); }
-#if MSORT_ABLATE & 8
-}  // namespace msort
-extern "C" void msort_debug_lb_stats(unsigned long long* out4, int reset) {
-    cudaMemcpyFromSymbol(out4, msort::g_lb_stats, 32);
-    if (reset) {
-        unsigned long long z[4] = {0, 0, 0, 0};
-        cudaMemcpyToSymbol(msort::g_lb_stats, z, 32);
-    }
-}
-namespace msort {
-#endif
+bool atomic_rank_ok(cudaStream_t caller) { return atomic_rank_ok_impl(caller); }
 
-uint32_t radix_tile_keys(int kt) { return key_bytes(kt) == 4 ? kMinTile32 : kMinTile64; }
+uint32_t radix_tile_keys(int kt) { return key_bytes(kt) == 4 ? Cfg32::kTile : Cfg64::kTile; }
+static uint32_t radix_group(int kt) { return key_bytes(kt) == 4 ? Cfg32::kGroup : Cfg64::kGroup; }
 
 static size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
 static size_t head_bytes() { return align_up(8 * 4 + 8 * 256 * 4 * 2 + 24 * 4, 256); }
 
-constexpr uint64_t kMinGroup = 8;  // smallest look-back group of the configs above (sizes the allocation)
-
-// look-back group size of the configuration in use (gagg stride; only that much is zeroed per sort)
-static uint64_t active_group(int kt) {
-    const int c = env_cfg();
-    uint32_t gsz;
-    if (key_bytes(kt) == 4) {
-        constexpr uint32_t G32[13] = {Cfg32_0::kGroup, Cfg32_1::kGroup, Cfg32_2::kGroup, Cfg32_3::kGroup, Cfg32_4::kGroup,
-                                      Cfg32_5::kGroup, Cfg32_6::kGroup, Cfg32_7::kGroup, Cfg32_8::kGroup, Cfg32_9::kGroup,
-                                      Cfg32_10::kGroup, Cfg32_11::kGroup, Cfg32_12::kGroup};
-        gsz = G32[c];
-    } else {
-        constexpr uint32_t G64[5] = {Cfg64_0::kGroup, Cfg64_1::kGroup, Cfg64_2::kGroup, Cfg64_3::kGroup, Cfg64_4::kGroup};
-        gsz = G64[c == 10 ? 4 : (c < 5 ? c : 0)];  // (11, 12: u32 only)
-    }
-    return gsz ? gsz : kMinGroup;
-}
-
-static uint64_t ws_groups(uint64_t tiles) { return tiles / kMinGroup + 1; }
-
+// Layout: head (counters, hist, bases, trivial) | group aggregates (zeroed per
+// sort) | status words (tagged, zeroed when the epoch wraps)
 size_t radix_ws_bytes(uint64_t n, int kt) {
     const uint64_t tiles = (n + radix_tile_keys(kt) - 1) / radix_tile_keys(kt);
-    return head_bytes() + align_up(size_t(tiles) * kRadix * 8, 256) +
-           size_t(num_passes(kt)) * ws_groups(tiles) * kRadix * 8 + 256;
+    const uint64_t groups = tiles / radix_group(kt) + 1;
+    const size_t garr = align_up(size_t(num_passes(kt)) * groups * kRadix * 8, 256);
+    return head_bytes() + garr + align_up(size_t(tiles) * kRadix * 8, 256) + 256;
 }
 
 RadixWs radix_ws_layout(void* ws, uint64_t n, int kt) {
@@ -843,12 +735,13 @@ RadixWs radix_ws_layout(void* ws, uint64_t n, int kt) {
     w.base = w.hist + 8 * 256;
     w.trivial = w.base + 8 * 256;
     w.head_bytes = head_bytes();
-    w.status = reinterpret_cast<unsigned long long*>(p + w.head_bytes);
     w.tiles = (n + radix_tile_keys(kt) - 1) / radix_tile_keys(kt);
-    w.groups = w.tiles / active_group(kt) + 1;  // <= ws_groups(tiles): the allocation covers any config
-    w.gagg = reinterpret_cast<unsigned long long*>(p + w.head_bytes + align_up(size_t(w.tiles) * kRadix * 8, 256));
-    w.zero_bytes = w.head_bytes + align_up(size_t(w.tiles) * kRadix * 8, 256) +
-                   size_t(num_passes(kt)) * w.groups * kRadix * 8;
+    w.groups = w.tiles / radix_group(kt) + 1;
+    const size_t garr = align_up(size_t(num_passes(kt)) * w.groups * kRadix * 8, 256);
+    w.gagg = reinterpret_cast<unsigned long long*>(p + w.head_bytes);
+    w.status = reinterpret_cast<unsigned long long*>(p + w.head_bytes + garr);
+    w.gagg_bytes = garr;
+    w.zero_bytes = w.head_bytes + garr + align_up(size_t(w.tiles) * kRadix * 8, 256);
     return w;
 }
 
@@ -887,13 +780,13 @@ cudaError_t launch_scan(const uint32_t* hist, uint32_t* base, uint32_t* trivial,
 cudaError_t radix_prologue(const void* keys, uint64_t n, int kt, const RadixWs& ws, cudaStream_t st) {
     cudaError_t e;
     if (ws.epoch == 0) {
-        e = cudaMemsetAsync(ws.counters, 0, ws.zero_bytes, st);
+        // a new tag cycle: no word of any earlier sort (of any size up to the
+        // allocation) may keep a tag that comes round again
+        e = cudaMemsetAsync(ws.counters, 0, ws.alloc_bytes > ws.zero_bytes ? ws.alloc_bytes : ws.zero_bytes, st);
     } else {
-        // epoch-tagged status words need no zeroing (1.1 GB at 4e9 keys); the
-        // per-pass tile counters and the group aggregates (atomic sums) do
-        e = cudaMemsetAsync(ws.counters, 0, ws.head_bytes, st);
-        if (e == cudaSuccess)
-            e = cudaMemsetAsync(ws.gagg, 0, size_t(num_passes(kt)) * ws.groups * kRadix * 8, st);
+        // tagged status words need no zeroing; the per-pass
+        // tile counters and the group aggregates (atomic sums) do
+        e = cudaMemsetAsync(ws.counters, 0, ws.head_bytes + ws.gagg_bytes, st);
     }
     if (e != cudaSuccess) return e;
     if ((e = launch_histogram(keys, n, kt, ws.hist, st)) != cudaSuccess) return e;

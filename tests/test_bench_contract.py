@@ -38,3 +38,50 @@ def test_reference_arm_under_torchrun_prints_once():
     assert r.returncode == 0, r.stderr[-2000:]
     lines = _lines(r.stdout)
     assert len(lines) == 1 and lines[0]["impl"] == "reference" and lines[0]["n_gpus"] == 2
+
+
+def _bench():
+    import importlib.util
+    spec = importlib.util.spec_from_file_location("bench_mod", os.path.join(ROOT, "bench.py"))
+    b = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(b)
+    return b
+
+
+def test_nvlink_fraction_fields():
+    """N > 1 lines carry the §8(d) S5 fractions: per Alg.2 stage the busiest mirrored pair's bytes over
+    the stage's exchange time, against 900 GB/s and against the in-run measured mirrored-pair peak."""
+    b = _bench()
+    st = {"stage_label": [2, 4, 2], "stage_max_x": [100, 0, 50], "stage_exchange_ms": [0.001, 0.0, 0.002]}
+    peaks = {"p2p_ce_gbs": 700.0, "p2p_sm_gbs": 800.0}
+    r = b.nvlink_fractions(st, 4, peaks, False)
+    assert {"per_stage", "achieved_gbs", "frac_of_900", "frac_of_measured_ce", "nominal_gbs", "measured_peaks",
+            "note"} <= set(r)
+    s0 = r["per_stage"][0]
+    assert s0["busiest_pair_bytes"] == 400 and abs(s0["achieved_gbs"] - 400 / 1e3) < 1e-12
+    assert abs(s0["frac_of_900"] - s0["achieved_gbs"] / 900) < 1e-12
+    assert abs(s0["frac_of_measured_ce"] - s0["achieved_gbs"] / 700) < 1e-12
+    assert r["per_stage"][1]["achieved_gbs"] is None          # a stage that moved nothing
+    assert "NVLink" in r["note"] and "HBM" in b.nvlink_fractions(st, 4, peaks, True)["note"]
+
+
+def test_output_verification_helpers():
+    """bench.py verifies the timed output: sorted under T and a permutation of the input."""
+    import numpy as np
+    import torch
+    import msort_inputs as mi
+    from oracle import sort as osort
+    b = _bench()
+    for kt in ("u32", "u64", "f32", "f64"):
+        a = mi.np_generate(5000, kt, "uniform", seed=3)
+        inp = torch.from_numpy(a.copy())
+        s = osort.oracle_sort(a, kt)
+        good = torch.from_numpy(s.copy())
+        r = b.verify_local(good, inp, len(a), kt, block=1024)
+        assert b.verify_all(r, None)["verified"], kt
+        x = s.copy()
+        x[[10, 20]] = x[[20, 10]]                               # unsorted
+        assert not b.verify_all(b.verify_local(torch.from_numpy(x), inp, len(a), kt, block=1024), None)["verified"], kt
+        y = s.copy()
+        y[-1] = y[-2]                                           # sorted, but not a permutation
+        assert not b.verify_all(b.verify_local(torch.from_numpy(y), inp, len(a), kt, block=1024), None)["verified"], kt

@@ -31,12 +31,13 @@ def _worker(rank, world, port, out_dir):
     import paper_conf_sigmod_maltenbergeritr22_b200 as m
     local = bytes([rank + 1]) * 7 + bytes(md.MSORT_DIST_HANDLE_BYTES - 7)
     allh = md.exchange_handles(local)
-    ch = md.chunking(1_000_003, world)
+    chunks = [m.msort_plan_chunk(1_000_003, world, r) for r in range(world)]
+    c = chunks[0][0]
     plans = []
     for s in range(m.msort_plan_num_stages(world)):
         label = m.msort_plan_stage(world, s)
-        piv = [(s * 7919 + j * 104729) % (ch.c * label // 2 + 1) for j in range(world // label)]
-        plans.append(m.msort_plan_exchange(world, s, ch.c, piv))
+        piv = [(s * 7919 + j * 104729) % (c * label // 2 + 1) for j in range(world // label)]
+        plans.append(m.msort_plan_exchange(world, s, c, piv))
     no_gpu_error = None
     if not torch.cuda.is_available():
         try:
@@ -45,7 +46,7 @@ def _worker(rank, world, port, out_dir):
             no_gpu_error = e.status
     np.save(os.path.join(out_dir, f"r{rank}.npy"), np.frombuffer(allh, dtype=np.uint8))
     with open(os.path.join(out_dir, f"r{rank}.txt"), "w") as f:
-        f.write(repr((ch.c, [ch.valid(r) for r in range(world)], plans, no_gpu_error)))
+        f.write(repr((c, chunks, plans, no_gpu_error)))
     dist.barrier()
     dist.destroy_process_group()
 
@@ -71,14 +72,23 @@ def test_dist_host_logic_gloo(tmp_path, world):
 
 
 def test_chunking_covers_input():
-    from paper_conf_sigmod_maltenbergeritr22_b200 import dist as md
-    for n in (0, 1, 7, 8, 9, 1000, 4_000_000_000):
+    """msort_plan_chunk (the library's chunking rule, include/msort.h) against the
+    oracle's reading Q3 (oracle.p2p.chunk_size): equal chunks of c keys, c a
+    multiple of 4, consecutive slices covering the n keys exactly once."""
+    import paper_conf_sigmod_maltenbergeritr22_b200 as m
+    from oracle import p2p
+    for n in (0, 1, 7, 8, 9, 1000, 65_537, 4_000_000_000, (1 << 32) + 3):
         for g in (1, 2, 4, 8):
-            ch = md.chunking(n, g)
-            assert ch.c % 4 == 0 and ch.c * g >= n
-            assert sum(ch.valid(r) for r in range(g)) == n
             seen = 0
             for r in range(g):
-                if ch.valid(r):
-                    assert ch.offset(r) == seen
-                    seen += ch.valid(r)
+                c, off, valid = m.msort_plan_chunk(n, g, r)
+                assert c == p2p.chunk_size(n, g) and c % 4 == 0 and c * g >= n
+                assert off == min(n, r * c) and 0 <= valid <= c
+                if valid:
+                    assert off == seen
+                seen += valid
+            assert seen == n
+    with pytest.raises(m.MsortError):
+        m.msort_plan_chunk(10, 3, 0)
+    with pytest.raises(m.MsortError):
+        m.msort_plan_chunk(10, 2, 2)

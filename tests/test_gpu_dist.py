@@ -26,7 +26,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, n, kt, distn, out_dir, host, exchange=0):
+def _worker(rank, world, port, n, kt, distn, out_dir, host, exchange=0, nccl=False):
     import sys
     sys.path.insert(0, ROOT)
     os.environ["MASTER_ADDR"] = "127.0.0.1"
@@ -36,26 +36,34 @@ def _worker(rank, world, port, n, kt, distn, out_dir, host, exchange=0):
     dist.init_process_group("gloo", rank=rank, world_size=world)
     import paper_conf_sigmod_maltenbergeritr22_b200 as m
     from paper_conf_sigmod_maltenbergeritr22_b200 import dist as md
-    ch = md.chunking(n, world)
-    ctx = md.dist_context(rank, world, 0, ch.c, kt)
+    c, off, v = m.msort_plan_chunk(n, world, rank)
+    try:
+        ctx = md.dist_context(rank, world, 0, c, kt, nccl=nccl)
+    except m.MsortError as e:
+        if nccl and e.status == 5:  # MSORT_ERR_NCCL: e.g. NCCL refuses two ranks on one GPU
+            with open(os.path.join(out_dir, f"nccl{rank}.txt"), "w") as f:
+                f.write(str(e))
+            dist.barrier()
+            dist.destroy_process_group()
+            return
+        raise
     ctx.set_option(m.MSORT_OPT_EXCHANGE, exchange)
     a = mi.np_generate(n, kt, distn, seed=5)
-    mine = np.full(ch.c, md.PAD_BITS[kt], dtype=codec.UINT[kt])
-    v = ch.valid(rank)
-    mine[:v] = codec.bits_of(a[ch.offset(rank):ch.offset(rank) + v], kt)
+    mine = codec.bits_of(a[off:off + v], kt).copy()   # this rank's slice; the library pads (reading Q3)
     if host:
         h = torch.from_numpy(mine.view(np.uint8).copy()).pin_memory()
-        ctx.sort_host(m.tensor_ptr(h), ch.c)
+        ctx.sort_host(m.tensor_ptr(h), n)
         res = h.numpy()
     else:
-        d = torch.from_numpy(mine.view(np.uint8).copy()).cuda()
-        ctx.sort(m.tensor_ptr(d), ch.c)
+        d = torch.zeros(c * mi.KEY_BYTES[kt], dtype=torch.uint8, device="cuda")
+        d[: v * mi.KEY_BYTES[kt]] = torch.from_numpy(mine.view(np.uint8).copy()).cuda()
+        ctx.sort(m.tensor_ptr(d), n)
         torch.cuda.synchronize()
-        res = d.cpu().numpy()
+        res = d[: v * mi.KEY_BYTES[kt]].cpu().numpy()
     np.save(os.path.join(out_dir, f"r{rank}.npy"), res)
     tm = ctx.timings()
     with open(os.path.join(out_dir, f"t{rank}.txt"), "w") as f:
-        f.write(repr(tm["stage_label"]))
+        f.write(repr((tm["stage_label"], tm["exchange_mode"], tm["peer_bulk_ok"])))
     ctx.close()
     dist.barrier()
     dist.destroy_process_group()
@@ -79,13 +87,30 @@ def _worker(rank, world, port, n, kt, distn, out_dir, host, exchange=0):
 def test_dist_sort_matches_oracle(tmp_path, world, n, kt, distn, host, exchange):
     mp.spawn(_worker, args=(world, _free_port(), n, kt, distn, str(tmp_path), host, exchange), nprocs=world,
              join=True)
-    from paper_conf_sigmod_maltenbergeritr22_b200 import dist as md
-    ch = md.chunking(n, world)
-    out = np.concatenate([np.load(tmp_path / f"r{r}.npy").view(codec.UINT[kt]) for r in range(world)])[:n]
+    out = np.concatenate([np.load(tmp_path / f"r{r}.npy").view(codec.UINT[kt]) for r in range(world)])
+    assert len(out) == n
     a = mi.np_generate(n, kt, distn, seed=5)
     assert np.array_equal(out, codec.bits_of(sort.oracle_sort(a, kt), kt))
-    labels = eval((tmp_path / "t0.txt").read_text())
-    assert len(labels) == (world - 1 if exchange < 2 else 1)
+    labels, mode, bulk_ok = eval((tmp_path / "t0.txt").read_text())
+    assert len(labels) == (world - 1 if exchange in (0, 1, 4) else 1)
+    assert bulk_ok == 1 and mode == exchange   # the peer bulk-copy self-test passed: no fallback
+
+
+def test_dist_nccl_swap(tmp_path):
+    """Exchange mode 4 in dist mode: an NCCL communicator bootstrapped from rank 0's
+    unique id (torch.distributed broadcast), grouped ncclSend/ncclRecv per
+    mirrored pair.  Two ranks on the test box's one GPU: if NCCL refuses that
+    (duplicate GPU), the refusal must come back as MSORT_ERR_NCCL, cleanly."""
+    world, n, kt = 2, 100_003, "u32"
+    mp.spawn(_worker, args=(world, _free_port(), n, kt, "uniform", str(tmp_path), False, 4, True), nprocs=world,
+             join=True)
+    refused = [(tmp_path / f"nccl{r}.txt").exists() for r in range(world)]
+    if all(refused):
+        pytest.skip("NCCL refused two ranks on one GPU: " + (tmp_path / "nccl0.txt").read_text()[:200])
+    assert not any(refused)
+    out = np.concatenate([np.load(tmp_path / f"r{r}.npy").view(codec.UINT[kt]) for r in range(world)])
+    a = mi.np_generate(n, kt, "uniform", seed=5)
+    assert np.array_equal(out, codec.bits_of(sort.oracle_sort(a, kt), kt))
 
 
 def _worker_big(rank, world, port, n, kt, distn, exchange, out_dir):
@@ -102,14 +127,9 @@ def _worker_big(rank, world, port, n, kt, distn, exchange, out_dir):
     import paper_conf_sigmod_maltenbergeritr22_b200 as m
     from paper_conf_sigmod_maltenbergeritr22_b200 import dist as md
     from oracle import checks
-    ch = md.chunking(n, world)
-    c, v = ch.c, ch.valid(rank)
+    c, off, v = m.msort_plan_chunk(n, world, rank)
     t = torch.empty(c, dtype=mi.torch_dtype(kt), device="cuda")
-    mi.t_generate_into(t[:v], n, kt, distn, seed=9, start=ch.offset(rank), block=1 << 27)
-    if v < c:  # reading Q3 padding (the largest key under T), as a signed bit pattern of the key width
-        signed = np.int32 if mi.KEY_BYTES[kt] == 4 else np.int64
-        pad = int(np.array([md.PAD_BITS[kt]], dtype=codec.UINT[kt]).view(signed)[0])
-        t.view(torch.int32 if mi.KEY_BYTES[kt] == 4 else torch.int64)[v:] = pad
+    mi.t_generate_into(t[:v], n, kt, distn, seed=9, start=off, block=1 << 27)
     blk = 1 << 26
 
     def fp(x, lim):
@@ -121,10 +141,9 @@ def _worker_big(rank, world, port, n, kt, distn, exchange, out_dir):
     fp_in = fp(t, v)
     ctx = md.dist_context(rank, world, 0, c, kt)
     ctx.set_option(m.MSORT_OPT_EXCHANGE, exchange)
-    ctx.sort(m.tensor_ptr(t), c)
+    ctx.sort(m.tensor_ptr(t), n)
     torch.cuda.synchronize()
-    # pads sort to the global end: the valid outputs are the first n of the concatenation
-    keep = max(0, min(c, n - rank * c))
+    keep = v  # this rank's sorted keys: global ranks [off, off + v)
     ok, first, last = True, None, None
     for off in range(0, keep, blk):
         codes = codec.encode(t[off:min(off + blk, keep)].cpu().numpy(), kt)

@@ -6,8 +6,8 @@ Together these imply byte equality with the (unique) oracle result.
 
 configs[2]: 4e9 uniform u32 on one GPU (the bench's N=1 workload);
 configs[1]: 2^28 uniform u32 on 2 chunks (virtual ranks on one GPU);
-configs[3]/[4]: 2e9 keys on 8 chunks (virtual ranks): zipf / reverse / nearly-sorted u32, f32, u64, and
-NEXT-1 on zipf.
+configs[3]/[4]: 2e9 keys on 8 chunks (virtual ranks): zipf / reverse / nearly-sorted / sorted / normal
+u32, f32, u64, NEXT-1 on zipf, and the NCCL swap (mode 4) on reverse.
 """
 import os
 
@@ -147,6 +147,9 @@ def test_config3_4e9_u32_one_gpu_end_to_end():
     (2_000_000_000, 8, "u32", "zipf", 0),        # configs[3] (pivot imbalance stress)
     (2_000_000_000, 8, "u32", "reverse", 0),     # configs[3]: x_d = c on every pair, every stage
     (2_000_000_000, 8, "u32", "nearly", 0),      # configs[3]
+    (2_000_000_000, 8, "u32", "sorted", 0),      # configs[3]: p = 0 every stage (no key moves)
+    (2_000_000_000, 8, "u32", "normal", 0),      # Fig.16's "normal" at g > 1
+    (2_000_000_000, 8, "u32", "reverse", 4),     # the NCCL send/recv swap (mode 4, self p2p on one GPU)
     (2_000_000_000, 8, "f32", "uniform", 0),     # configs[4] float keys
     (2_000_000_000, 8, "u64", "uniform", 0),     # configs[4] 64-bit keys
     (2_000_000_000, 8, "u32", "zipf", 2),        # NEXT-1 (fused all-to-all) at full size

@@ -71,6 +71,26 @@ def test_repeated_sorts_one_context(ms, g):
     ctx.close()
 
 
+def test_epoch_wrap_zeroes_whole_workspace(ms):
+    """the look-back words carry an epoch tag that comes round again
+    after 512 sorts; when the epoch wraps to 0 the WHOLE workspace is zeroed, so
+    a large sort at epoch E, a small one across the wrap, and a large one at
+    epoch E again must all be right (stale E-tagged words past the small sort's
+    tiles would otherwise be read as published)."""
+    big, small = 4 * 300_000, 4 * 1000
+    ctx = ms.Context(1, big, "u32", device_ids=[0])
+    ctx.set_option(ms.MSORT_OPT_SMALL_GRAPH, 0)
+    E = 300
+    for i, (n, before) in enumerate([(big, E - 1), (small, 511), (big, E - 1), (small, 511), (big, E - 1)]):
+        ctx.set_option(ms.MSORT_OPT_RADIX_EPOCH, before)
+        a = mi.np_generate(n, "u32", ["uniform", "zipf"][i % 2], seed=40 + i)
+        d = dev_keys(a)
+        ctx.sort_device([ms.tensor_ptr(d)], n)
+        torch.cuda.synchronize()
+        assert np.array_equal(host_keys(d, "u32"), sort.oracle_sort(a, "u32")), (i, n)
+    ctx.close()
+
+
 @pytest.mark.parametrize("dist", mi.DISTRIBUTIONS)
 def test_radix_sort_distributions(ms, dist):
     n = 3 * (1 << 18) + 77
@@ -246,7 +266,7 @@ def _virtual_sort(ms, a, kt, g, exchange=0):
 
 
 @pytest.mark.parametrize("g", [2, 4, 8])
-@pytest.mark.parametrize("dist", ["uniform", "sorted", "reverse", "nearly", "zipf"])
+@pytest.mark.parametrize("dist", ["uniform", "sorted", "reverse", "nearly", "zipf", "normal"])
 def test_p2p_sort_virtual_ranks(ms, g, dist):
     c = 3 * 7680 + 44
     a = mi.np_generate(g * c, "u32", dist, seed=g)
@@ -259,6 +279,80 @@ def test_p2p_sort_virtual_ranks(ms, g, dist):
     for s, st in enumerate(stages):
         assert tm["stage_pivot"][s][: len(st)] == [op.p for op in st]
         assert tm["stage_max_x"][s] == max(max(op.xs) for op in st)
+
+
+def _staged_chunks(ms, a, kt, g, exchange, stop):
+    """Virtual-rank Alg.2 stopped after stage `stop` (MSORT_OPT_STOP_AFTER_STAGE): every chunk."""
+    n = len(a)
+    c = n // g
+    ctx = ms.Context(g, n, kt, device_ids=[0] * g)
+    ctx.set_option(ms.MSORT_OPT_EXCHANGE, exchange)
+    ctx.set_option(ms.MSORT_OPT_STOP_AFTER_STAGE, stop)
+    chunks = [dev_keys(a[i * c:(i + 1) * c]) for i in range(g)]
+    ctx.sort_device([ms.tensor_ptr(t) for t in chunks], c)
+    torch.cuda.synchronize()
+    out = [host_keys(t, kt) for t in chunks]
+    tm = ctx.timings()
+    ctx.close()
+    return out, tm
+
+
+@pytest.mark.parametrize("exchange", [0, 1, 4])
+@pytest.mark.parametrize("g", [2, 4, 8])
+@pytest.mark.parametrize("dist", ["uniform", "reverse", "dups", "zipf"])
+def test_alg2_every_stage_matches_stage_model(ms, g, dist, exchange):
+    """SURVEY §8(c) S7 pin: after EVERY Alg.2 stage, every GPU's chunk equals the
+    oracle's stage model (oracle.p2p.run_stages, Alg.2 P:1804-1818 in its
+    concurrent form, reading Q7) - the fused device-resident exchange (0), the
+    paper's copy-then-merge swap (1) and the NCCL send/recv swap (4)."""
+    c = 2 * 4864 + 52   # several merge tiles and a ragged one
+    if dist == "dups":
+        a = (mi.np_generate(g * c, "u32", "uniform", seed=g + 3) % np.uint32(97)).astype(np.uint32)
+    else:
+        a = mi.np_generate(g * c, "u32", dist, seed=g + 3)
+    codes = [np.sort(codec.encode(a[i * c:(i + 1) * c], "u32")) for i in range(g)]
+    stages = p2p.run_stages(codes)
+    for s, st in enumerate(stages):
+        expect = [None] * g
+        for op in st:
+            for k, ch in enumerate(op.after):
+                expect[op.lo + k] = ch
+        out, tm = _staged_chunks(ms, a, "u32", g, exchange, s)
+        assert tm["n_stages"] == s + 1
+        assert tm["stage_pivot"][s][: len(st)] == [op.p for op in st]
+        for q in range(g):
+            assert np.array_equal(out[q], expect[q]), (s, q)
+
+
+@pytest.mark.parametrize("exchange", [0, 1, 4])
+@pytest.mark.parametrize("c", [1, 3, 5003, 4864 + 1])
+def test_p2p_sort_ragged_chunks(ms, c, exchange):
+    """Chunks whose size is not a multiple of 4 keys (a ragged tail after the last
+    16-byte unit) through every Alg.2 exchange mode."""
+    g = 4
+    a = mi.np_generate(g * c, "u32", "uniform", seed=c)
+    out, _ = _virtual_sort(ms, a, "u32", g, exchange=exchange)
+    assert np.array_equal(out, sort.oracle_sort(a, "u32"))
+
+
+@pytest.mark.parametrize("g", [2, 4, 8])
+@pytest.mark.parametrize("dist", ["uniform", "sorted", "reverse", "zipf"])
+def test_p2p_sort_nccl_swap(ms, g, dist):
+    """Exchange mode 4: the swap as grouped ncclSend/ncclRecv per mirrored pair (one
+    communicator on the one GPU: NCCL self send/recv), then the local merge."""
+    c = 3 * 7680 + 44
+    a = mi.np_generate(g * c, "u32", dist, seed=g + 11)
+    out, tm = _virtual_sort(ms, a, "u32", g, exchange=4)
+    assert np.array_equal(out, sort.oracle_sort(a, "u32"))
+    assert tm["stage_label"] == p2p.stage_labels(g)
+
+
+@pytest.mark.parametrize("kt", ["u64", "f32", "f64"])
+def test_p2p_sort_nccl_swap_key_types(ms, kt):
+    g, c = 4, 5003
+    a = mi.np_generate(g * c, kt, "uniform", seed=23)
+    out, _ = _virtual_sort(ms, a, kt, g, exchange=4)
+    assert np.array_equal(bits(out, kt), bits(sort.oracle_sort(a, kt), kt))
 
 
 @pytest.mark.parametrize("kt", ["u64", "f32", "f64"])
