@@ -617,6 +617,28 @@ __global__ void __launch_bounds__(256) rank_probe_kernel(uint32_t seed, uint32_t
     }
 }
 
+// production-configuration check (below): 0 = equal, 1 = mismatch, -1 = could not run
+int production_rank_check(cudaStream_t ps);
+
+// Keys for the production check: many equal pass-1 digits (3 bits of byte 1),
+// random low byte, so stability is what decides the order of equal digits.
+__global__ void rank_check_keys(uint32_t* k32, uint64_t* k64, uint32_t n, uint32_t seed) {
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+        uint32_t h = (i + 1) * 0x9E3779B9u ^ seed;
+        h ^= h >> 16;
+        h *= 0x85EBCA6Bu;
+        h ^= h >> 13;
+        const uint32_t key = (h & 0xFFFF00FFu) | (((h >> 8) & 7u) << 8);
+        k32[i] = key;
+        k64[i] = (uint64_t(h * 0xC2B2AE35u) << 32) | key;
+    }
+}
+
+__global__ void count_diff(const uint32_t* a, const uint32_t* b, uint64_t words, uint32_t* bad) {
+    for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < words; i += uint64_t(gridDim.x) * blockDim.x)
+        if (a[i] != b[i]) atomicAdd(bad, 1u);
+}
+
 // The probe runs once per device on a private stream, outside any capture:
 // called while the caller's stream (or this thread) is capturing a CUDA graph
 // it answers "no" for this call only (the conservative peer-match ranking) and
@@ -651,6 +673,12 @@ bool atomic_rank_ok_impl(cudaStream_t caller) {
         if (cudaGetLastError() == cudaSuccess && cudaMemcpyAsync(&hb, bad, 4, cudaMemcpyDeviceToHost, ps) == cudaSuccess &&
             cudaStreamSynchronize(ps) == cudaSuccess)
             verdict = hb == 0 ? 1 : -1;
+        // and the production kernels themselves: one stable pass with atomic
+        // ranking must equal the same pass with peer-match ranking, byte for byte
+        if (verdict == 1) {
+            const int pc = production_rank_check(ps);
+            verdict = pc == 0 ? 1 : (pc > 0 ? -1 : 0);
+        }
     }
     if (bad) cudaFree(bad);
     if (ps) cudaStreamDestroy(ps);
@@ -806,5 +834,56 @@ cudaError_t launch_onesweep(const void* in, void* out, uint64_t n, int kt, int p
         default: return cudaErrorInvalidValue;
     }
 }
+
+namespace {
+
+template <typename U>
+int production_check_t(cudaStream_t ps, U* keys, U* out_a, U* out_b, void* ws_mem, size_t ws_bytes, uint32_t n,
+                       uint32_t* bad) {
+    const int kt = sizeof(U) == 4 ? 0 : 1;
+    RadixWs ws = radix_ws_layout(ws_mem, n, kt);
+    ws.epoch = 0;
+    auto ok = [](cudaError_t e) { return e == cudaSuccess; };
+    for (int stable = 0; stable < 2; ++stable) {
+        if (!ok(cudaMemsetAsync(ws_mem, 0, ws_bytes, ps)) || !ok(radix_prologue(keys, n, kt, ws, ps))) return -1;
+        // pass 1 (digit = byte 1): flags 4 = atomic ranking, 0 = peer match
+        if (!ok(launch_onesweep(keys, stable ? out_b : out_a, n, kt, 1, stable ? 0 : 4, ws, ws.base + 256, ps)))
+            return -1;
+    }
+    count_diff<<<148, 256, 0, ps>>>(reinterpret_cast<const uint32_t*>(out_a), reinterpret_cast<const uint32_t*>(out_b),
+                                    uint64_t(n) * sizeof(U) / 4, bad);
+    return cudaGetLastError() == cudaSuccess ? 0 : -1;
+}
+
+int production_rank_check(cudaStream_t ps) {
+    const uint32_t n = 6 * Cfg32::kTile + 1237;  // several tiles and a ragged one (both key widths)
+    uint32_t* k32 = nullptr;
+    uint64_t* k64 = nullptr;
+    void* outs = nullptr;
+    void* ws = nullptr;
+    uint32_t* bad = nullptr;
+    const size_t wsb = std::max(radix_ws_bytes(n, 0), radix_ws_bytes(n, 1));
+    int rc = -1;
+    if (cudaMalloc(&k32, n * 4ull) == cudaSuccess && cudaMalloc(&k64, n * 8ull) == cudaSuccess &&
+        cudaMalloc(&outs, n * 16ull) == cudaSuccess && cudaMalloc(&ws, wsb) == cudaSuccess &&
+        cudaMalloc(&bad, 4) == cudaSuccess && cudaMemsetAsync(bad, 0, 4, ps) == cudaSuccess) {
+        rank_check_keys<<<148, 256, 0, ps>>>(k32, k64, n, 0x6A09E667u);
+        char* o = static_cast<char*>(outs);
+        if (production_check_t<uint32_t>(ps, k32, reinterpret_cast<uint32_t*>(o), reinterpret_cast<uint32_t*>(o + n * 4ull),
+                                         ws, wsb, n, bad) == 0 &&
+            production_check_t<uint64_t>(ps, k64, reinterpret_cast<uint64_t*>(o), reinterpret_cast<uint64_t*>(o + n * 8ull),
+                                         ws, wsb, n, bad) == 0) {
+            uint32_t hb = 1;
+            if (cudaMemcpyAsync(&hb, bad, 4, cudaMemcpyDeviceToHost, ps) == cudaSuccess && cudaStreamSynchronize(ps) == cudaSuccess)
+                rc = hb == 0 ? 0 : 1;
+        }
+    }
+    for (void* p : {static_cast<void*>(k32), static_cast<void*>(k64), outs, ws, static_cast<void*>(bad)})
+        if (p) cudaFree(p);
+    cudaGetLastError();
+    return rc;
+}
+
+}  // namespace
 
 }  // namespace msort

@@ -7,8 +7,10 @@ import paper_conf_sigmod_maltenbergeritr22_b200 as ms
 from oracle import sort as osort
 def dev(a): return torch.from_numpy(a.view(np.uint8).copy()).cuda()
 ok = True
+# (g > 1, mode 0: the device-resident Alg.2 stages; mode 4: the NCCL send/recv swap; 4 x 5003: ragged chunks)
 for kt, n, g, ex in [("u32", 20011, 1, 0), ("f32", 30000, 4, 0), ("u64", 9001 * 2, 2, 1), ("u32", 24000, 4, 2),
-                     ("u64", 16000, 8, 2), ("u32", 24000, 4, 3)]:
+                     ("u64", 16000, 8, 2), ("u32", 24000, 4, 3), ("u32", 4 * 5003, 4, 0), ("u32", 32000, 8, 0),
+                     ("u32", 4 * 5003, 4, 4), ("f64", 12000, 2, 4)]:
     a = mi.np_generate(n, kt, "uniform", seed=2)
     c = n // g
     ctx = ms.Context(g, n, kt, device_ids=[0] * g)
@@ -56,4 +58,16 @@ for kt, oa, ob, oo, al, bl in [("u32", 1, 3, 2, 9001, 7777), ("u64", 1, 0, 1, 50
     good = np.array_equal(got.view(np.uint8), osort.oracle_sort(np.concatenate([a, b]), kt).view(np.uint8))
     ok &= good
     print("merge", kt, al, bl, "ok" if good else "MISMATCH", flush=True)
+# interconnect measurement and the out-of-core HET baseline (NEXT-4)
+ctx = ms.Context(2, 1 << 20, "u32", device_ids=[0, 0])
+print("links", ctx.measure_links(1 << 20, 1), flush=True)
+ctx.close()
+from baseline import het
+a = mi.np_generate(300_001, "u32", "uniform", seed=9)
+h = torch.from_numpy(a.copy()).pin_memory()
+o = torch.empty_like(h)
+het.het_ooc_sort(h, "u32", 1 << 16, [0, 0], o)
+good = np.array_equal(o.numpy(), osort.oracle_sort(a, "u32"))
+ok &= good
+print("het ooc", "ok" if good else "MISMATCH", flush=True)
 print("ALL OK" if ok else "FAIL")
