@@ -80,6 +80,8 @@ def parse(argv=None):
                          "GPUs; 2 NEXT-1 (P:3416-3424) single all-to-all fused into the merge; 3 NEXT-1 pull then "
                          "merge. The other of {0, 2} is timed too and reported beside it")
     ap.add_argument("--no-compare", action="store_true", help="N>1: skip the second merge-phase variant")
+    ap.add_argument("--no-nccl", action="store_true",
+                    help="N>1: skip the NCCL send/recv swap (exchange mode 4) leg (only runs on distinct GPUs)")
     ap.add_argument("--het", action="store_true", help="also time the HET-sort baseline (GPU chunk sorts + CPU merge)")
     ap.add_argument("--het-chunks", type=int, default=8)
     ap.add_argument("--het-gpus", type=int, default=0, help="GPUs for the HET chunk sorts (0: all visible)")
@@ -335,7 +337,8 @@ def verify_all(local, dist):
 # --- interconnect fractions ---------------------------------------------------------------------------------
 
 def nvlink_fractions(stages: dict, K: int, peaks: dict | None, same_device: bool):
-    """Per merge stage: busiest mirrored pair's bytes / the stage's exchange time."""
+    """Per merge stage: busiest mirrored pair's bytes / the stage's exchange time (fused modes: the
+    exchange+merge kernel; copy / NCCL modes: pass the transfer-only time as stage_exchange_ms)."""
     rows = []
     for s, (lab, mx, ms) in enumerate(zip(stages["stage_label"], stages["stage_max_x"], stages["stage_exchange_ms"])):
         b = mx * K
@@ -488,6 +491,34 @@ def main():
                    "verified": v2["verified"]}
         ctx.set_option(ms.MSORT_OPT_EXCHANGE, args.exchange)
 
+    # --- N>1 on distinct GPUs: the swap as NCCL send/recv (mode 4, the north star's S5 mechanism)
+    nccl_leg = None
+    if g > 1 and not args.no_nccl:
+        if same_gpu:
+            nccl_leg = {"unavailable": "ranks share one GPU (NCCL refuses two ranks of a communicator on one device)"}
+        else:
+            try:
+                obj = [ms.msort_nccl_unique_id() if rank == 0 else None]
+                dist.broadcast_object_list(obj, src=0)
+                ctx.nccl_init(obj[0])
+                ctx.set_option(ms.MSORT_OPT_EXCHANGE, 4)
+                for _ in range(2):
+                    with torch.cuda.stream(stream):
+                        work.copy_(pristine)
+                    sort_dev()
+                barrier()
+                r4 = timed_steps(args.steps)
+                v4 = verify_all(verify_local(work, pristine, valid, kt), dist)
+                t4 = r4["tm"]
+                st4 = {"stage_label": t4["stage_label"], "stage_max_x": t4["stage_max_x"],
+                       "stage_exchange_ms": [max_over_ranks(x) for x in t4["stage_swap_ms"]]}
+                nccl_leg = {"value": n / (r4["ms_per_step"] / 1e3), "unit": "keys/s", "ms_per_step": r4["ms_per_step"],
+                            "exchange": "Alg.2, swap as grouped ncclSend/ncclRecv per mirrored pair, then local merge",
+                            "verified": v4["verified"], "swap_stage_ms": st4["stage_exchange_ms"], "stages": st4}
+            except ms.MsortError as e:
+                nccl_leg = {"unavailable": str(e)}
+            ctx.set_option(ms.MSORT_OPT_EXCHANGE, args.exchange)
+
     # --- interconnect peaks (msort_measure_links; every rank, collective in dist mode)
     peaks = None
     if not args.no_links:
@@ -541,6 +572,11 @@ def main():
         st = {k: stage_info[k] for k in ("stage_label", "stage_max_x")}
         st["stage_exchange_ms"] = [max_over_ranks(x) for x in stage_info["stage_exchange_ms"]]
         nvlink = nvlink_fractions(st, K, peaks if peaks and "error" not in peaks else None, same_gpu)
+        nvlink["time_basis"] = "fused exchange+merge kernel time per stage (the partner's block is read inside the merge)"
+        if nccl_leg and "stages" in nccl_leg:
+            nccl_leg["nvlink"] = nvlink_fractions(nccl_leg.pop("stages"), K,
+                                                  peaks if peaks and "error" not in peaks else None, same_gpu)
+            nccl_leg["nvlink"]["time_basis"] = "ncclSend/ncclRecv group time per stage (transfer only)"
 
     # --- end to end through the public host API
     e2e = None
@@ -638,7 +674,7 @@ def main():
                           "merge_phase": merge_phase_ms},
             "stages": {k: stage_info[k] for k in ("stage_label", "stage_pivot", "stage_max_x", "stage_ms",
                                                   "stage_exchange_ms")} if stage_info and g > 1 else None,
-            "nvlink": nvlink, "links": peaks,
+            "nvlink": nvlink, "links": peaks, "nccl_swap": nccl_leg,
             "paper_context": PAPER_CONTEXT,
             "het_baseline": het,
             ("next1" if args.exchange == 0 else "alg2"): compare,

@@ -179,6 +179,8 @@ typedef struct {
     int      peer_bulk_ok;                              /* 1: TMA bulk copies from peer memory passed the
                                                            self-test msort_create / msort_dist_import run
                                                            between distinct devices (or none needed)   */
+    double   stage_swap_ms[MSORT_MAX_STAGES];           /* the transfer alone (modes 1 / 4: copy or NCCL
+                                                           send/recv; fused modes: = stage_exchange_ms) */
 } msort_timings;
 
 int msort_get_timings(const msort_ctx* ctx, msort_timings* out);

@@ -166,6 +166,7 @@ struct Rank {
     cudaEvent_t e_nccl[2] = {};  // exchange mode 4: ranks sharing a device hand their stream to one NCCL stream
     cudaEvent_t e_stage[MSORT_MAX_STAGES][2] = {};
     cudaEvent_t e_xch[MSORT_MAX_STAGES][2] = {};
+    cudaEvent_t e_swp[MSORT_MAX_STAGES] = {};  // modes 1 / 4: end of the transfer (the merge follows)
     bool xch_rec[MSORT_MAX_STAGES] = {};  // e_xch[s] recorded in this sort
     // per sort
     void* user = nullptr;
@@ -265,6 +266,7 @@ int alloc_rank(msort_ctx* ctx, Rank& R, bool need_b1, bool need_stage) {
         for (auto& e : se) CUDA_TRY(cudaEventCreate(&e));
     for (auto& xe : R.e_xch)
         for (auto& e : xe) CUDA_TRY(cudaEventCreate(&e));
+    for (auto& e : R.e_swp) CUDA_TRY(cudaEventCreate(&e));
     return MSORT_OK;
 }
 
@@ -301,6 +303,8 @@ void free_rank(Rank& R) {
     for (auto& xe : R.e_xch)
         for (auto e : xe)
             if (e) cudaEventDestroy(e);
+    for (auto e : R.e_swp)
+        if (e) cudaEventDestroy(e);
     for (auto e : R.e_piece)
         if (e) cudaEventDestroy(e);
     for (auto e : R.e_slice)
@@ -429,12 +433,15 @@ int launch_exchange(msort_ctx* ctx, Rank& R, int stage, bool last, uint64_t c, u
     void* out = R.ptr(out_idx);
     // (mode 4 recorded the start before the NCCL swap)
     if (ctx->timing && ctx->xmode != 4) CUDA_TRY(cudaEventRecord(R.e_xch[stage][0], R.st));
+    const bool swp = ctx->timing && (ctx->xmode == 1 || ctx->xmode == 4);
     if (x == c) {
         // the whole chunk moves: a pure P2P copy (one sorted run, reading Q8);
         // mode 4 received it into `out` already
         if (ctx->xmode != 4) CUDA_TRY(cudaMemcpyAsync(out, peer, c * K, cudaMemcpyDefault, R.st));
+        if (swp) CUDA_TRY(cudaEventRecord(R.e_swp[stage], R.st));
     } else if (ctx->xmode == 4) {
         // NCCL swap done (nccl_stage_exchange): the partner's block is in B2
+        if (swp) CUDA_TRY(cudaEventRecord(R.e_swp[stage], R.st));
         const char* recv = static_cast<const char*>(R.buf[2]);
         if (side == 0)
             CUDA_TRY(launch_merge(ownb, c - x, recv, x, out, ctx->kt, R.mws, R.st, &ctx->tm.kernel_launches));
@@ -451,9 +458,11 @@ int launch_exchange(msort_ctx* ctx, Rank& R, int stage, bool last, uint64_t c, u
         char* recv = static_cast<char*>(R.buf[2]);
         if (side == 0) {
             CUDA_TRY(cudaMemcpyAsync(recv, peerb, x * K, cudaMemcpyDefault, R.st));
+            if (swp) CUDA_TRY(cudaEventRecord(R.e_swp[stage], R.st));
             CUDA_TRY(launch_merge(ownb, c - x, recv, x, out, ctx->kt, R.mws, R.st, &ctx->tm.kernel_launches));
         } else {
             CUDA_TRY(cudaMemcpyAsync(recv, peerb + (c - x) * K, x * K, cudaMemcpyDefault, R.st));
+            if (swp) CUDA_TRY(cudaEventRecord(R.e_swp[stage], R.st));
             CUDA_TRY(launch_merge(recv, x, ownb + x * K, c - x, out, ctx->kt, R.mws, R.st, &ctx->tm.kernel_launches));
         }
     }
@@ -1407,14 +1416,18 @@ static void collect_exchange_timings(msort_ctx* ctx) {
     if (!ctx->timing) return;
     // e_xch events are recorded only on ranks that exchanged in that stage
     for (int s = 0; s < ctx->tm.n_stages; ++s) {
-        double mx = 0;
+        double mx = 0, sw = 0;
         for (int i = 0; i < ctx->nlocal; ++i) {
             Rank& R = ctx->r[i];
             if (!R.xch_rec[s]) continue;
             cudaSetDevice(R.dev);
             mx = std::max(mx, double(elapsed(R.e_xch[s][0], R.e_xch[s][1])));
+            if (ctx->xmode == 1 || ctx->xmode == 4)
+                sw = std::max(sw, double(elapsed(R.e_xch[s][0], R.e_swp[s])));
         }
         ctx->tm.stage_exchange_ms[s] = mx;
+        // the transfer alone: separate in modes 1 / 4, the same as the exchange when fused (modes 0, 2)
+        ctx->tm.stage_swap_ms[s] = (ctx->xmode == 1 || ctx->xmode == 4) ? sw : mx;
     }
 }
 

@@ -345,6 +345,10 @@ def test_p2p_sort_nccl_swap(ms, g, dist):
     out, tm = _virtual_sort(ms, a, "u32", g, exchange=4)
     assert np.array_equal(out, sort.oracle_sort(a, "u32"))
     assert tm["stage_label"] == p2p.stage_labels(g)
+    assert tm["exchange_mode"] == 4
+    for mx, sw, ex in zip(tm["stage_max_x"], tm["stage_swap_ms"], tm["stage_exchange_ms"]):
+        if mx:  # the NCCL transfer alone is timed, and it is part of the stage's exchange + merge
+            assert 0 < sw <= ex
 
 
 @pytest.mark.parametrize("kt", ["u64", "f32", "f64"])
@@ -517,3 +521,35 @@ def test_rank_mode_probe(ms):
     mode = ms.msort_rank_mode(0)
     assert mode in (0, 1)
     print("onesweep ranking:", "atomic (lane-ordered)" if mode == 1 else "peer match")
+
+
+def test_soak_mixed_sizes_one_context(ms):
+    """Stress of the cross-block protocols racecheck cannot see (the global-memory
+    decoupled look-back with epoch-tagged status words, the device-resident merge
+    stages): 120 back-to-back sorts in two long-lived contexts with random sizes
+    around tile and group boundaries, random distributions and key types, each
+    equal to the oracle."""
+    rng = np.random.default_rng(2024)
+    cap = 1 << 21
+    ctxs = {g: ms.Context(g, cap, "u32", device_ids=[0] * g) for g in (1, 4)}
+    ctxs[1].set_option(ms.MSORT_OPT_SMALL_GRAPH, 0)
+    for it in range(120):
+        g = 1 if it % 3 else 4
+        tiles = int(rng.integers(1, (cap // g) // 7168))
+        c = max(4, tiles * 7168 + int(rng.integers(-300, 300))) // 4 * 4
+        dist = ["uniform", "zipf", "sorted", "reverse", "nearly", "normal"][int(rng.integers(0, 6))]
+        a = mi.np_generate(g * c, "u32", dist, seed=it)
+        chunks = [dev_keys(a[i * c:(i + 1) * c]) for i in range(g)]
+        ctxs[g].sort_device([ms.tensor_ptr(t) for t in chunks], c)
+        torch.cuda.synchronize()
+        got = np.concatenate([host_keys(t, "u32") for t in chunks])
+        assert np.array_equal(got, sort.oracle_sort(a, "u32")), (it, g, c, dist)
+    for c in ctxs.values():
+        c.close()
+
+
+def test_rank_mode_is_atomic_on_b200(ms):
+    """On sm_100 the lane-order probe AND the production-kernel check (one stable pass
+    with atomic ranking equals the same pass with peer-match ranking, both key widths)
+    pass, so the passes rank with one shared atomic per key (reading Q16)."""
+    assert ms.msort_rank_mode(0) == 1
