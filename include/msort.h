@@ -82,9 +82,10 @@ typedef enum {
  *            to a multiple of 4) keys; the tail is padded with the largest key
  *            under T and the padding is dropped (reading Q3).
  *   stream   the sort is ordered after work already queued on `stream`; the call
- *            BLOCKS until the sorted result is in `keys` (NCCL-free host round
- *            trips per merge stage make the call synchronous anyway).
- * A per-(device set, key type) context is cached and grown on demand. */
+ *            BLOCKS until the sorted result is in `keys` (the statistics of the
+ *            merge stages are read back at the end).
+ * A per-(device set, key type) context is cached and grown on demand
+ * (msort_release_cached drops them). */
 int msort_sort(void* keys, uint64_t n, int key_type, int n_gpus, void* stream);
 
 /* ------------------------------------------------------------------------ */
