@@ -34,6 +34,10 @@ CONFIGS = [  # (BASELINE.json configs index, n, g, key type, distribution, excha
     (4, 2_000_000_000, 8, "u64", "uniform", 2),
     (4, 2_000_000_000, 8, "f32", "uniform", 0),
     (4, 2_000_000_000, 8, "f32", "uniform", 2),
+    (1, 1 << 28, 2, "u32", "uniform", 1),        # the paper's copy-then-merge swap
+    (1, 1 << 28, 2, "u32", "uniform", 4),        # the NCCL send/recv swap (self p2p on one GPU)
+    (3, 2_000_000_000, 8, "u32", "reverse", 4),
+    (3, 2_000_000_000, 8, "u32", "normal", 0),
 ]
 only = os.environ.get("CONFIGS")
 for idx, n, g, kt, dist, ex in CONFIGS:
@@ -63,7 +67,9 @@ for idx, n, g, kt, dist, ex in CONFIGS:
     print(json.dumps({"config": idx, "n": n, "g": g, "kt": kt, "dist": dist, "exchange": ex, "ms": ms_avg,
                       "keys_per_s": n / (ms_avg / 1e3), "sort_ms": tm["sort_ms"], "merge_ms": tm["merge_ms"],
                       "stage_label": tm["stage_label"], "stage_max_x": tm["stage_max_x"],
-                      "stage_ms": [round(x, 3) for x in tm["stage_ms"]], "virtual_ranks": g > 1}), flush=True)
+                      "stage_ms": [round(x, 3) for x in tm["stage_ms"]],
+                      "stage_swap_ms": [round(x, 3) for x in tm["stage_swap_ms"]],
+                      "exchange_mode_run": tm["exchange_mode"], "virtual_ranks": g > 1}), flush=True)
     ctx.close()
     del src, work
     torch.cuda.empty_cache()
