@@ -186,6 +186,22 @@ class ClockSampler:
                 "samples": len(self.rows), "source": "nvml" if self.nv is not None else "nvidia-smi"}
 
 
+class stdout_to_stderr:
+    """fd-level redirect of stdout to stderr (NCCL prints its version line on stdout at init; the bench's
+    stdout carries exactly one JSON line)."""
+
+    def __enter__(self):
+        sys.stdout.flush()
+        self.saved = os.dup(1)
+        os.dup2(2, 1)
+        return self
+
+    def __exit__(self, *a):
+        sys.stdout.flush()
+        os.dup2(self.saved, 1)
+        os.close(self.saved)
+
+
 def cpu_model() -> str:
     try:
         with open("/proc/cpuinfo") as f:
@@ -498,9 +514,10 @@ def main():
             nccl_leg = {"unavailable": "ranks share one GPU (NCCL refuses two ranks of a communicator on one device)"}
         else:
             try:
-                obj = [ms.msort_nccl_unique_id() if rank == 0 else None]
-                dist.broadcast_object_list(obj, src=0)
-                ctx.nccl_init(obj[0])
+                with stdout_to_stderr():
+                    obj = [ms.msort_nccl_unique_id() if rank == 0 else None]
+                    dist.broadcast_object_list(obj, src=0)
+                    ctx.nccl_init(obj[0])
                 ctx.set_option(ms.MSORT_OPT_EXCHANGE, 4)
                 for _ in range(2):
                     with torch.cuda.stream(stream):
