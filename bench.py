@@ -510,14 +510,22 @@ def main():
     # --- N>1 on distinct GPUs: the swap as NCCL send/recv (mode 4, the north star's S5 mechanism)
     nccl_leg = None
     if g > 1 and not args.no_nccl:
-        if same_gpu:
+        if same_gpu and os.environ.get("MSORT_BENCH_FORCE_NCCL") != "1":  # (=1: exercise the refusal path)
             nccl_leg = {"unavailable": "ranks share one GPU (NCCL refuses two ranks of a communicator on one device)"}
         else:
+            err = None
             try:
                 with stdout_to_stderr():
                     obj = [ms.msort_nccl_unique_id() if rank == 0 else None]
                     dist.broadcast_object_list(obj, src=0)
                     ctx.nccl_init(obj[0])
+            except Exception as e:  # (collective decision below: every rank runs the leg or none does)
+                err = str(e)
+            okt = torch.tensor([0 if err else 1], dtype=torch.int32)
+            dist.all_reduce(okt, op=dist.ReduceOp.MIN)
+            if int(okt.item()) == 0:
+                nccl_leg = {"unavailable": err or "NCCL init failed on another rank"}
+            else:
                 ctx.set_option(ms.MSORT_OPT_EXCHANGE, 4)
                 for _ in range(2):
                     with torch.cuda.stream(stream):
@@ -532,8 +540,6 @@ def main():
                 nccl_leg = {"value": n / (r4["ms_per_step"] / 1e3), "unit": "keys/s", "ms_per_step": r4["ms_per_step"],
                             "exchange": "Alg.2, swap as grouped ncclSend/ncclRecv per mirrored pair, then local merge",
                             "verified": v4["verified"], "swap_stage_ms": st4["stage_exchange_ms"], "stages": st4}
-            except ms.MsortError as e:
-                nccl_leg = {"unavailable": str(e)}
             ctx.set_option(ms.MSORT_OPT_EXCHANGE, args.exchange)
 
     # --- interconnect peaks (msort_measure_links; every rank, collective in dist mode)
