@@ -172,13 +172,20 @@ int het_ooc_sort(void* host_keys, uint64_t n, int key_type, int g, const int* de
     double t0 = now_s(), t1 = t0, t2 = t0;
     if (rc == 0) {
         std::vector<int> rcs(g, 0);
+        std::vector<std::string> errs(g);
         std::vector<std::thread> th;
         char* host = static_cast<char*>(host_keys);
         for (int i = 0; i < g; ++i)
-            th.emplace_back([&, i]() { rcs[i] = run_gpu(gs[i], host, n, ck, K, key_type, i, g, &runs[i]); });
+            th.emplace_back([&, i]() {
+                rcs[i] = run_gpu(gs[i], host, n, ck, K, key_type, i, g, &runs[i]);
+                errs[i] = g_err;  // (g_err is per thread: hand it to the caller's thread)
+            });
         for (auto& t : th) t.join();
-        for (int r : rcs)
-            if (r) rc = r;
+        for (int i = 0; i < g; ++i)
+            if (rcs[i] && !rc) {
+                rc = rcs[i];
+                g_err = errs[i];
+            }
         t1 = now_s();
     }
     std::vector<std::pair<uint64_t, uint64_t>> all;

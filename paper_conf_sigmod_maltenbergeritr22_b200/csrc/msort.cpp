@@ -1343,8 +1343,8 @@ int msort_create(msort_ctx** out, int n_gpus, const int* device_ids, uint64_t ma
         }
     }
     if (n_gpus > 1) {
-        const int s = peer_bulk_selftest_local(ctx.get());
-        if (s == MSORT_OK) apply_exchange_mode(ctx.get());
+        int s = peer_bulk_selftest_local(ctx.get());
+        if (s == MSORT_OK) s = apply_exchange_mode(ctx.get());
         if (s != MSORT_OK) {
             for (int j = 0; j < n_gpus; ++j) free_rank(ctx->r[j]);
             return s;

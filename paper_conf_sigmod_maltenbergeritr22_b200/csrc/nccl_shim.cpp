@@ -51,7 +51,8 @@ void load_api() {
         if (h) break;
     }
     if (!h) {
-        g_api.err = std::string("dlopen libnccl.so.2 failed: ") + (dlerror() ? dlerror() : "?");
+        const char* why = dlerror();  // (dlerror clears the message: read it once)
+        g_api.err = std::string("dlopen libnccl.so.2 failed: ") + (why ? why : "?");
         return;
     }
     bool ok = sym(h, "ncclGetUniqueId", g_api.GetUniqueId) && sym(h, "ncclCommInitRank", g_api.CommInitRank) &&
