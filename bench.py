@@ -85,6 +85,9 @@ def parse(argv=None):
     ap.add_argument("--het", action="store_true", help="also time the HET-sort baseline (GPU chunk sorts + CPU merge)")
     ap.add_argument("--het-chunks", type=int, default=8)
     ap.add_argument("--het-gpus", type=int, default=0, help="GPUs for the HET chunk sorts (0: all visible)")
+    ap.add_argument("--het-ooc-chunk", type=float, default=0,
+                    help="also time the out-of-core HET sort (NEXT-4, 2n-approach) with chunks of this many keys "
+                         "(two chunk buffers per GPU: a device budget below the input)")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--cpu-parallel-keys", type=float, default=float(1 << 28))
     return ap.parse_args(argv)
@@ -676,6 +679,28 @@ def main():
                "gpu_sort_and_copies_s": info["gpu_sort_and_copies_s"], "cpu_merge_s": info["cpu_merge_s"]}
         del hk, src, hs
 
+    het_ooc = None
+    if args.het_ooc_chunk and g == 1:
+        from baseline import het as hetmod
+        ngpu = torch.cuda.device_count() if args.het_gpus <= 0 else min(args.het_gpus, torch.cuda.device_count())
+        hk = torch.empty(n, dtype=tdt, pin_memory=True)
+        ho = torch.empty(n, dtype=tdt, pin_memory=True)
+        src = pristine[:n].cpu()
+        ck = int(args.het_ooc_chunk)
+        hk.copy_(src)
+        hetmod.het_ooc_sort(hk, kt, ck, list(range(ngpu)), ho)     # warm-up (OpenMP start, allocations)
+        hk.copy_(src)
+        info = hetmod.het_ooc_sort(hk, kt, ck, list(range(ngpu)), ho)
+        ok = bool(torch.equal(ho[:min(n, 1 << 20)].view(torch.uint8), work[:min(n, 1 << 20)].cpu().view(torch.uint8)))
+        het_ooc = {"value": n / info["total_s"], "unit": "keys/s",
+                   "kind": f"out-of-core HET (paper §5.3 2n-approach, NEXT-4) on {ngpu} GPU(s): chunks of {ck} keys, "
+                           f"two chunk buffers per GPU ({2 * ck * K / 2**30:.1f} GiB), CPU multiway merge "
+                           f"({info['threads']} threads)",
+                   "chunks": info["chunks"], "chunk_groups": info["chunk_groups"],
+                   "gpu_phase_s": info["gpu_phase_s"], "cpu_merge_s": info["merge_s"],
+                   "prefix_matches_device_sort": ok}
+        del hk, ho, src
+
     merge_phase_ms = max_over_ranks(stage_info["merge_ms"]) if stage_info else None
     if rank == 0:
         out = {
@@ -699,7 +724,7 @@ def main():
                                                   "stage_exchange_ms")} if stage_info and g > 1 else None,
             "nvlink": nvlink, "links": peaks, "nccl_swap": nccl_leg,
             "paper_context": PAPER_CONTEXT,
-            "het_baseline": het,
+            "het_baseline": het, "het_out_of_core": het_ooc,
             ("next1" if args.exchange == 0 else "alg2"): compare,
         }
         print(json.dumps(out))
