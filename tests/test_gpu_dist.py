@@ -26,19 +26,20 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, n, kt, distn, out_dir, host, exchange=0, nccl=False):
+def _worker(rank, world, port, n, kt, distn, out_dir, host, exchange=0, nccl=False, distinct=False):
     import sys
     sys.path.insert(0, ROOT)
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     os.environ.setdefault("MSORT_BARRIER_TIMEOUT_S", "120")
-    torch.cuda.set_device(0)
+    dev = rank if distinct else 0
+    torch.cuda.set_device(dev)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     import paper_conf_sigmod_maltenbergeritr22_b200 as m
     from paper_conf_sigmod_maltenbergeritr22_b200 import dist as md
     c, off, v = m.msort_plan_chunk(n, world, rank)
     try:
-        ctx = md.dist_context(rank, world, 0, c, kt, nccl=nccl)
+        ctx = md.dist_context(rank, world, dev, c, kt, nccl=nccl)
     except m.MsortError as e:
         if nccl and e.status == 5:  # MSORT_ERR_NCCL: e.g. NCCL refuses two ranks on one GPU
             with open(os.path.join(out_dir, f"nccl{rank}.txt"), "w") as f:
@@ -55,8 +56,8 @@ def _worker(rank, world, port, n, kt, distn, out_dir, host, exchange=0, nccl=Fal
         ctx.sort_host(m.tensor_ptr(h), n)
         res = h.numpy()
     else:
-        d = torch.zeros(c * mi.KEY_BYTES[kt], dtype=torch.uint8, device="cuda")
-        d[: v * mi.KEY_BYTES[kt]] = torch.from_numpy(mine.view(np.uint8).copy()).cuda()
+        d = torch.zeros(c * mi.KEY_BYTES[kt], dtype=torch.uint8, device=f"cuda:{dev}")
+        d[: v * mi.KEY_BYTES[kt]] = torch.from_numpy(mine.view(np.uint8).copy()).to(f"cuda:{dev}")
         ctx.sort(m.tensor_ptr(d), n)
         torch.cuda.synchronize()
         res = d[: v * mi.KEY_BYTES[kt]].cpu().numpy()
@@ -181,3 +182,21 @@ def test_dist_sort_full_size(tmp_path, world, n, kt, distn, exchange):
             f = [f[0] + r[k][0], (f[1] + r[k][1]) % (1 << 64), f[2] ^ r[k][2]]
         return f
     assert tot("fp_in") == tot("fp_out") and tot("fp_in")[0] == n
+
+
+@pytest.mark.parametrize("exchange", [0, 2, 4])
+def test_dist_sort_distinct_gpus(tmp_path, exchange):
+    """One process per GPU on distinct GPUs (skipped on one-GPU boxes): IPC over NVLink, device barriers,
+    the NCCL communicator of mode 4 - equal to the oracle."""
+    world = min(torch.cuda.device_count(), 8)
+    world = 1 << (world.bit_length() - 1) if world else 0
+    if world < 2:
+        pytest.skip("needs 2 or more GPUs")
+    n, kt = 1_000_003, "u32"
+    mp.spawn(_worker, args=(world, _free_port(), n, kt, "uniform", str(tmp_path), False, exchange, exchange == 4, True),
+             nprocs=world, join=True)
+    out = np.concatenate([np.load(tmp_path / f"r{r}.npy").view(codec.UINT[kt]) for r in range(world)])
+    a = mi.np_generate(n, kt, "uniform", seed=5)
+    assert np.array_equal(out, codec.bits_of(sort.oracle_sort(a, kt), kt))
+    labels, mode, bulk_ok = eval((tmp_path / "t0.txt").read_text())
+    assert bulk_ok == 1 and mode == exchange

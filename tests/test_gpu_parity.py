@@ -553,3 +553,34 @@ def test_rank_mode_is_atomic_on_b200(ms):
     with atomic ranking equals the same pass with peer-match ranking, both key widths)
     pass, so the passes rank with one shared atomic per key (reading Q16)."""
     assert ms.msort_rank_mode(0) == 1
+
+
+# ---------------------------------------------------------------------------
+# Distinct GPUs (skipped on one-GPU boxes): the same paths over NVLink
+# ---------------------------------------------------------------------------
+
+@pytest.mark.parametrize("exchange", [0, 1, 2, 4])
+@pytest.mark.parametrize("g", [2, 4, 8])
+def test_p2p_sort_distinct_gpus(ms, g, exchange):
+    """Chunk i on GPU i (peer access over NVLink): every exchange mode equals the oracle, every Alg.2 stage
+    equals the stage model, and the peer bulk-copy self-test ran between distinct devices."""
+    if torch.cuda.device_count() < g:
+        pytest.skip(f"needs {g} GPUs")
+    c = 2 * 7168 + 36
+    a = mi.np_generate(g * c, "u32", "uniform", seed=g * 10 + exchange)
+    ctx = ms.Context(g, g * c, "u32", device_ids=list(range(g)))
+    ctx.set_option(ms.MSORT_OPT_EXCHANGE, exchange)
+    chunks = [torch.from_numpy(a[i * c:(i + 1) * c].view(np.uint8).copy()).to(f"cuda:{i}") for i in range(g)]
+    ctx.sort_device([ms.tensor_ptr(t) for t in chunks], c)
+    for i in range(g):
+        torch.cuda.synchronize(i)
+    out = np.concatenate([t.cpu().numpy().view(np.uint32) for t in chunks])
+    tm = ctx.timings()
+    assert np.array_equal(out, sort.oracle_sort(a, "u32"))
+    assert tm["peer_bulk_ok"] == 1 and tm["exchange_mode"] == exchange
+    if exchange in (0, 1, 4):
+        codes = [np.sort(a[i * c:(i + 1) * c]) for i in range(g)]
+        stages = p2p.run_stages(codes)
+        for s, st in enumerate(stages):
+            assert tm["stage_pivot"][s][: len(st)] == [op.p for op in st]
+    ctx.close()
