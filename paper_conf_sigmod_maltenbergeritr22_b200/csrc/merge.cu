@@ -173,9 +173,11 @@ __global__ void __launch_bounds__(256) splitter_kernel(GroupPtrs all, int g, uin
     }
 }
 
-// Same partition, one THREAD per boundary (plain binary search): the top levels
-// of all searches hit the same L2 lines, so DRAM sees only the last few levels
-// of each search (the warp version above touches 64 sectors per round).
+// Merge-path partition: part[t] = number of a-elements among the first
+// min(t*tile, total) outputs (a wins ties), one THREAD per boundary (plain
+// binary search): the top levels of all searches hit the same L2 lines, so DRAM
+// sees only the last few levels of each search (a warp-wide 32-ary search per
+// boundary, round 1, touched 64 sectors per round and was slower).
 // dyn != nullptr: the runs and their lengths come from device memory (the
 // device-resident Alg.2 stage, resolved on the GPU after the pivot search).
 template <typename U, bool FLOAT>
@@ -210,7 +212,7 @@ __global__ void __launch_bounds__(256) partition_thread_kernel(const U* __restri
 // one output tile's A range followed by its B range (na + nb = TILE keys, plus
 // alignment slack), so 3 blocks x (STAGES-1) tiles of input are in flight per
 // SM (Little's law at ~6.5 TB/s x ~1.5 us HBM / NVLink latency needs ~65 KB per
-// SM; the two-stage kernel above keeps <= 45 KB).  Every range is bulk-copied
+// SM; round 1's two-stage version kept <= 45 KB).  Every range is bulk-copied
 // from its 16-byte-aligned start to the 16-byte boundary after its end: the
 // over-fetch never leaves the 16-byte units that hold the range's own first and
 // last keys, so it cannot cross a page, and no thread-issued tail loads remain
