@@ -611,11 +611,8 @@ int selftest_merge(msort_ctx* ctx, Rank& R, const void* peer_odd, uint32_t n, bo
     CUDA_TRY(cudaMemcpyAsync(got.data(), R.buf[1], (2 * n - 1) * 4, cudaMemcpyDeviceToHost, R.st));
     CUDA_TRY(cudaStreamSynchronize(R.st));
     bool good = true;
-    for (uint32_t k = 0, t = 0; k < 2 * n - 1; ++k) {  // expected: 0, 2, 3, 4, 5, ... (odd 1 skipped)
-        const uint32_t want = k == 0 ? 0 : k + 1;
-        good = good && got[k] == want;
-        (void)t;
-    }
+    for (uint32_t k = 0; k < 2 * n - 1; ++k)  // expected: 0, 2, 3, 4, 5, ... (the odd 1 is skipped)
+        good = good && got[k] == (k == 0 ? 0 : k + 1);
     *ok = good;
     return MSORT_OK;
 }
