@@ -200,3 +200,48 @@ def test_dist_sort_distinct_gpus(tmp_path, exchange):
     assert np.array_equal(out, codec.bits_of(sort.oracle_sort(a, kt), kt))
     labels, mode, bulk_ok = eval((tmp_path / "t0.txt").read_text())
     assert bulk_ok == 1 and mode == exchange
+
+
+def _worker_soak(rank, world, port, out_dir, iters):
+    """Many back-to-back dist sorts of random sizes, distributions and exchange modes in ONE context per
+    rank: the device barriers (release/acquire on IPC-mapped flags), the epoch-tagged look-back and the
+    device-resident stages under repeated reuse of the same buffers."""
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    os.environ.setdefault("MSORT_BARRIER_TIMEOUT_S", "120")
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import paper_conf_sigmod_maltenbergeritr22_b200 as m
+    from paper_conf_sigmod_maltenbergeritr22_b200 import dist as md
+    cap = 1 << 19
+    ctx = md.dist_context(rank, world, 0, cap, "u32")
+    rng = np.random.default_rng(77)          # the same sequence on every rank
+    bad = []
+    for it in range(iters):
+        n = int(rng.integers(world, world * cap))
+        distn = ["uniform", "zipf", "reverse", "sorted", "nearly"][int(rng.integers(0, 5))]
+        ex = [0, 1, 2, 3][int(rng.integers(0, 4))]
+        ctx.set_option(m.MSORT_OPT_EXCHANGE, ex)
+        c, off, v = m.msort_plan_chunk(n, world, rank)
+        a = mi.np_generate(n, "u32", distn, seed=it)
+        d = torch.zeros(c, dtype=torch.int32, device="cuda")
+        d[:v] = torch.from_numpy(a[off:off + v].view(np.int32).copy()).cuda()
+        ctx.sort(m.tensor_ptr(d), n)
+        torch.cuda.synchronize()
+        want = sort.oracle_sort(a, "u32")[off:off + v]
+        if not np.array_equal(d[:v].cpu().numpy().view(np.uint32), want):
+            bad.append((it, n, distn, ex))
+    with open(os.path.join(out_dir, f"soak{rank}.txt"), "w") as f:
+        f.write(repr(bad))
+    ctx.close()
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_dist_soak(tmp_path):
+    world, iters = 4, 40
+    mp.spawn(_worker_soak, args=(world, _free_port(), str(tmp_path), iters), nprocs=world, join=True)
+    for r in range(world):
+        assert (tmp_path / f"soak{r}.txt").read_text() == "[]", r
