@@ -250,6 +250,9 @@ struct OsCfg {
 #ifndef MSORT_G64
 #define MSORT_G64 16
 #endif
+#ifndef MSORT_LB_SLEEP_NS
+#define MSORT_LB_SLEEP_NS 32  // back-off of a look-back poll on an unpublished predecessor
+#endif
 #define MSORT_CFG32 OsCfg<MSORT_T32, MSORT_I32, 0x5555555u, MSORT_B32, MSORT_W32, MSORT_G32, true>
 #define MSORT_CFG64 OsCfg<256, 14, 0x1555u, 4, MSORT_W64, MSORT_G64, false>
 using Cfg32 = MSORT_CFG32;
@@ -360,7 +363,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
                 if (used == 0) {
                     unsigned long long w;
                     do {
-                        __nanosleep(32);
+                        __nanosleep(MSORT_LB_SLEEP_NS);
                         w = ld_relaxed_gpu(p);
                     } while (uint32_t(w >> 32) != hi_agg && uint32_t(w >> 32) != hi_incl);
                 }
@@ -398,7 +401,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
                     }
                     if (done || used == h + 1) break;  // (all groups down to 0 consumed)
                     h -= used;
-                    if (used == 0) __nanosleep(32);
+                    if (used == 0) __nanosleep(MSORT_LB_SLEEP_NS);
                 }
             }
             st_relaxed_gpu(&status[uint64_t(tile) * kRadix + d], pack_status(kFlagIncl, tag, excl + my_total));
