@@ -228,7 +228,7 @@ struct OsCfg {
 // may override single parameters with -DMSORT_W32=4 etc.):
 //   u32/f32: 7168-key tiles, 4 blocks of 256 threads per SM, look-back window 2,
 //            groups of 32, next tile counted after the scatter (3 barriers)
-//   u64/f64: 3584-key tiles, 4 blocks per SM, window 4, groups of 16
+//   u64/f64: 3584-key tiles, 4 blocks per SM, window 1, groups of 16
 #ifndef MSORT_T32
 #define MSORT_T32 256
 #endif
@@ -245,7 +245,7 @@ struct OsCfg {
 #define MSORT_G32 32
 #endif
 #ifndef MSORT_W64
-#define MSORT_W64 4
+#define MSORT_W64 1  // round 2: 8.24 ms per 2e9-key u64 pass vs 8.45 at window 4 (profiles/radix_tuning_r2.md)
 #endif
 #ifndef MSORT_G64
 #define MSORT_G64 16
