@@ -254,7 +254,10 @@ struct OsCfg {
 #define MSORT_LB_SLEEP_NS 32  // back-off of a look-back poll on an unpublished predecessor
 #endif
 #define MSORT_CFG32 OsCfg<MSORT_T32, MSORT_I32, 0x5555555u, MSORT_B32, MSORT_W32, MSORT_G32, true>
-#define MSORT_CFG64 OsCfg<256, 14, 0x1555u, 4, MSORT_W64, MSORT_G64, false>
+#ifndef MSORT_CE64
+#define MSORT_CE64 false  // (counting the next tile after the scatter: 3% slower for 8-byte keys in round 1)
+#endif
+#define MSORT_CFG64 OsCfg<256, 14, 0x1555u, 4, MSORT_W64, MSORT_G64, MSORT_CE64>
 using Cfg32 = MSORT_CFG32;
 using Cfg64 = MSORT_CFG64;
 template <typename U>
