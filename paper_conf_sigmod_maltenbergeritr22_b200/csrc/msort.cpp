@@ -23,8 +23,10 @@
 #include <cstring>
 #include <map>
 #include <memory>
+#include <condition_variable>
 #include <mutex>
 #include <string>
+#include <thread>
 #include <tuple>
 #include <vector>
 
@@ -164,6 +166,9 @@ struct Rank {
     bool small_seen = false;
     cudaEvent_t e_sync[MSORT_MAX_STAGES + 1] = {};
     cudaEvent_t e_nccl[2] = {};  // exchange mode 4: ranks sharing a device hand their stream to one NCCL stream
+    // pageable host memory (S0/S8): pinned bounce buffers, allocated on first use
+    void* bounce[3] = {nullptr, nullptr, nullptr};
+    cudaEvent_t e_bounce[3] = {};
     cudaEvent_t e_stage[MSORT_MAX_STAGES][2] = {};
     cudaEvent_t e_xch[MSORT_MAX_STAGES][2] = {};
     cudaEvent_t e_swp[MSORT_MAX_STAGES] = {};  // modes 1 / 4: end of the transfer (the merge follows)
@@ -310,6 +315,10 @@ void free_rank(Rank& R) {
     for (auto e : R.e_slice)
         if (e) cudaEventDestroy(e);
     if (R.e_merged) cudaEventDestroy(R.e_merged);
+    for (void* b : R.bounce)
+        if (b) cudaFreeHost(b);
+    for (auto e : R.e_bounce)
+        if (e) cudaEventDestroy(e);
     if (R.small_exec) cudaGraphExecDestroy(R.small_exec);
     if (R.cst) {
         cudaStreamSynchronize(R.cst);
@@ -561,6 +570,133 @@ int nccl_stage_exchange(msort_ctx* ctx, const Exchange& ex, uint64_t c, bool las
         CUDA_TRY(cudaSetDevice(ctx->r[l].dev));
         CUDA_TRY(cudaEventRecord(ctx->r[l].e_nccl[1], ctx->r[l].st));
         CUDA_TRY(cudaStreamWaitEvent(ctx->r[i].st, ctx->r[l].e_nccl[1], 0));
+    }
+    return MSORT_OK;
+}
+
+// --- pageable host memory (S0 / S8) -----------------------------------------------
+// A copy from pageable memory makes the driver stage it through its own small
+// pinned buffers one piece at a time (measured: 4e9 u32 keys, msort_sort on a
+// numpy array 2.21 s vs 0.57 s pinned).  Pageable host keys go through a ring
+// of pinned bounce buffers per GPU instead: host threads copy chunk k into a
+// bounce buffer while the copy engine moves chunk k-1 (H2D), or the copy engine
+// fills chunk k+1 while the threads drain chunk k (D2H), so PCIe stays busy.
+constexpr size_t kBounceBytes = size_t(64) << 20;
+constexpr int kBounce = 3;
+
+class CopyPool {  // parallel memcpy on the host cores (persistent workers)
+  public:
+    static CopyPool& get() {
+        static CopyPool* p = new CopyPool;  // (never destroyed: its detached workers wait on it until exit)
+        return *p;
+    }
+    void copy(void* dst, const void* src, size_t bytes) {
+        std::lock_guard<std::mutex> one(call_mu_);  // one copy at a time (contexts may live on several threads)
+        const int parts = int(std::min<size_t>(workers_.size() + 1, std::max<size_t>(1, bytes >> 20)));
+        if (parts <= 1) {
+            std::memcpy(dst, src, bytes);
+            return;
+        }
+        const size_t step = (bytes + parts - 1) / parts;
+        {
+            std::lock_guard<std::mutex> lk(mu_);
+            dst_ = static_cast<char*>(dst);
+            src_ = static_cast<const char*>(src);
+            bytes_ = bytes;
+            step_ = step;
+            pending_ = parts - 1;
+            jobs_ = parts - 1;
+        }
+        cv_.notify_all();
+        std::memcpy(dst, src, std::min(step, bytes));  // the caller copies part 0
+        std::unique_lock<std::mutex> lk(mu_);
+        done_.wait(lk, [&] { return pending_ == 0; });
+    }
+
+  private:
+    CopyPool() {
+        const unsigned hw = std::thread::hardware_concurrency();
+        const int n = int(std::min<unsigned>(15, hw > 1 ? hw - 1 : 1));
+        for (int i = 0; i < n; ++i) workers_.emplace_back([this] { loop(); });
+        for (auto& t : workers_) t.detach();  // (live for the process)
+    }
+    void loop() {
+        for (;;) {
+            std::unique_lock<std::mutex> lk(mu_);
+            cv_.wait(lk, [&] { return jobs_ > 0; });
+            const int part = jobs_--;  // parts P-1 .. 1 of the current copy
+            char* d = dst_;
+            const char* s = src_;
+            const size_t step = step_, bytes = bytes_;
+            lk.unlock();
+            const size_t off = size_t(part) * step;
+            if (off < bytes) std::memcpy(d + off, s + off, std::min(step, bytes - off));
+            lk.lock();
+            if (--pending_ == 0) done_.notify_all();
+        }
+    }
+    std::vector<std::thread> workers_;
+    std::mutex call_mu_, mu_;
+    std::condition_variable cv_, done_;
+    char* dst_ = nullptr;
+    const char* src_ = nullptr;
+    size_t bytes_ = 0, step_ = 0;
+    int pending_ = 0, jobs_ = 0;
+};
+
+bool host_is_pageable(const void* p) {
+    cudaPointerAttributes a{};
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return true;
+    }
+    return a.type == cudaMemoryTypeUnregistered;
+}
+
+int bounce_alloc(Rank& R) {
+    if (R.bounce[0]) return MSORT_OK;
+    CUDA_TRY(cudaSetDevice(R.dev));
+    for (int b = 0; b < kBounce; ++b) {
+        CUDA_TRY(cudaMallocHost(&R.bounce[b], kBounceBytes));
+        CUDA_TRY(cudaEventCreateWithFlags(&R.e_bounce[b], cudaEventDisableTiming));
+    }
+    return MSORT_OK;
+}
+
+// pageable host -> device through the bounce ring (returns when every chunk is queued)
+int bounce_h2d(Rank& R, void* dst, const char* src, size_t bytes, cudaStream_t st) {
+    MSORT_TRY(bounce_alloc(R));
+    char* d = static_cast<char*>(dst);
+    for (size_t off = 0, k = 0; off < bytes; off += kBounceBytes, ++k) {
+        const int b = int(k % kBounce);
+        const size_t len = std::min(kBounceBytes, bytes - off);
+        if (k >= size_t(kBounce)) CUDA_TRY(cudaEventSynchronize(R.e_bounce[b]));  // its last DMA is done
+        CopyPool::get().copy(R.bounce[b], src + off, len);
+        CUDA_TRY(cudaMemcpyAsync(d + off, R.bounce[b], len, cudaMemcpyHostToDevice, st));
+        CUDA_TRY(cudaEventRecord(R.e_bounce[b], st));
+    }
+    return MSORT_OK;
+}
+
+// device -> pageable host through the bounce ring (returns when the data is in `dst`)
+int bounce_d2h(Rank& R, char* dst, const void* src, size_t bytes, cudaStream_t st) {
+    MSORT_TRY(bounce_alloc(R));
+    const char* sp = static_cast<const char*>(src);
+    const size_t nch = (bytes + kBounceBytes - 1) / kBounceBytes;
+    auto issue = [&](size_t k) -> int {
+        const int b = int(k % kBounce);
+        const size_t off = k * kBounceBytes, len = std::min(kBounceBytes, bytes - off);
+        CUDA_TRY(cudaMemcpyAsync(R.bounce[b], sp + off, len, cudaMemcpyDeviceToHost, st));
+        CUDA_TRY(cudaEventRecord(R.e_bounce[b], st));
+        return MSORT_OK;
+    };
+    for (size_t k = 0; k < std::min<size_t>(nch, kBounce); ++k) MSORT_TRY(issue(k));
+    for (size_t k = 0; k < nch; ++k) {
+        const int b = int(k % kBounce);
+        const size_t off = k * kBounceBytes, len = std::min(kBounceBytes, bytes - off);
+        CUDA_TRY(cudaEventSynchronize(R.e_bounce[b]));
+        CopyPool::get().copy(dst + off, R.bounce[b], len);
+        if (k + kBounce < nch) MSORT_TRY(issue(k + kBounce));
     }
     return MSORT_OK;
 }
@@ -1590,7 +1726,9 @@ int msort_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n) {
     reset_timings(ctx, c);
     const size_t K = key_bytes(ctx->kt);
     char* host = static_cast<char*>(host_keys);
-    if (g == 1 && ctx->host_pipeline && c >= kPipeMinKeys) return sort_host_pipelined(ctx, host, n, c);
+    // pageable keys: through pinned bounce buffers (no transfer/sort overlap, but PCIe rate)
+    const bool pageable = host_is_pageable(host_keys);
+    if (g == 1 && ctx->host_pipeline && c >= kPipeMinKeys && !pageable) return sort_host_pipelined(ctx, host, n, c);
     for (int i = 0; i < g; ++i) {
         Rank& R = ctx->r[i];
         CUDA_TRY(cudaSetDevice(R.dev));
@@ -1599,7 +1737,8 @@ int msort_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n) {
         const uint64_t lo = std::min<uint64_t>(n, uint64_t(i) * c);
         const uint64_t cnt = std::min<uint64_t>(n - lo, c);
         CUDA_TRY(cudaEventRecord(R.e_h2d0, R.st));
-        if (cnt) CUDA_TRY(cudaMemcpyAsync(R.stage, host + lo * K, cnt * K, cudaMemcpyHostToDevice, R.st));
+        if (cnt && pageable) MSORT_TRY(bounce_h2d(R, R.stage, host + lo * K, cnt * K, R.st));
+        else if (cnt) CUDA_TRY(cudaMemcpyAsync(R.stage, host + lo * K, cnt * K, cudaMemcpyHostToDevice, R.st));
         CUDA_TRY(launch_fill_max(static_cast<char*>(R.stage) + cnt * K, c - cnt, ctx->kt, R.st));
         if (c > cnt) ctx->tm.kernel_launches += 1;
         CUDA_TRY(cudaEventRecord(R.e_h2d1, R.st));
@@ -1611,7 +1750,8 @@ int msort_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n) {
         const uint64_t lo = std::min<uint64_t>(n, uint64_t(i) * c);
         const uint64_t cnt = std::min<uint64_t>(n - lo, c);
         CUDA_TRY(cudaEventRecord(R.e_d2h0, R.st));
-        if (cnt) CUDA_TRY(cudaMemcpyAsync(host + lo * K, R.stage, cnt * K, cudaMemcpyDeviceToHost, R.st));
+        if (cnt && pageable) MSORT_TRY(bounce_d2h(R, host + lo * K, R.stage, cnt * K, R.st));
+        else if (cnt) CUDA_TRY(cudaMemcpyAsync(host + lo * K, R.stage, cnt * K, cudaMemcpyDeviceToHost, R.st));
         CUDA_TRY(cudaEventRecord(R.e_d2h1, R.st));
     }
     for (int i = 0; i < g; ++i) {
@@ -2019,17 +2159,20 @@ int msort_dist_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n_total) {
     CUDA_TRY(cudaSetDevice(R.dev));
     reset_timings(ctx, c);
     const size_t K = key_bytes(ctx->kt);
-    if (ctx->host_pipeline && c >= kPipeMinKeys) {
+    const bool pageable = valid && host_is_pageable(host_keys);
+    if (ctx->host_pipeline && c >= kPipeMinKeys && !pageable) {
         // pipelined S0 (MSORT_OPT_HOST_PIPELINE): H2D pieces sorted as they land (the pad is filled there)
         MSORT_TRY(dist_sort_impl(ctx, R.stage, c, R.st, true, static_cast<const char*>(host_keys), valid));
     } else {
         CUDA_TRY(cudaEventRecord(R.e_h2d0, R.st));
-        if (valid) CUDA_TRY(cudaMemcpyAsync(R.stage, host_keys, valid * K, cudaMemcpyHostToDevice, R.st));
+        if (pageable) MSORT_TRY(bounce_h2d(R, R.stage, static_cast<const char*>(host_keys), valid * K, R.st));
+        else if (valid) CUDA_TRY(cudaMemcpyAsync(R.stage, host_keys, valid * K, cudaMemcpyHostToDevice, R.st));
         CUDA_TRY(cudaEventRecord(R.e_h2d1, R.st));
         MSORT_TRY(dist_sort_impl(ctx, R.stage, c, R.st, true, nullptr, valid));
     }
     CUDA_TRY(cudaEventRecord(R.e_d2h0, R.st));
-    if (valid) CUDA_TRY(cudaMemcpyAsync(host_keys, R.stage, valid * K, cudaMemcpyDeviceToHost, R.st));
+    if (pageable) MSORT_TRY(bounce_d2h(R, static_cast<char*>(host_keys), R.stage, valid * K, R.st));
+    else if (valid) CUDA_TRY(cudaMemcpyAsync(host_keys, R.stage, valid * K, cudaMemcpyDeviceToHost, R.st));
     CUDA_TRY(cudaEventRecord(R.e_d2h1, R.st));
     CUDA_TRY(cudaEventSynchronize(R.e_d2h1));
     ctx->tm.h2d_ms = elapsed(R.e_h2d0, R.e_h2d1);

@@ -445,6 +445,22 @@ def test_msort_sort_host_pointer(ms, n, kt):
     assert bits(h, kt).tobytes() == bits(sort.oracle_sort(a, kt), kt).tobytes()
 
 
+@pytest.mark.parametrize("n,kt,g", [(50_000_003, "u32", 1), (20_000_001, "f64", 2), (33_554_437, "u64", 4)])
+def test_pageable_host_bounce(ms, n, kt, g):
+    """Pageable host keys (numpy) spanning several 64 MiB pinned bounce buffers: the host threads' copies,
+    the bounce ring's events and the padding of the last chunk, through msort_sort (the north-star entry,
+    g = 1) and a context (virtual ranks)."""
+    a = mi.np_generate(n, kt, "uniform", seed=n % 97)
+    h = a.copy()
+    if g == 1:
+        ms.msort_sort(h.ctypes.data, n, kt, 1)
+    else:
+        ctx = ms.Context(g, n, kt, device_ids=[0] * g)
+        ctx.sort_host(h.ctypes.data, n)
+        ctx.close()
+    assert bits(h, kt).tobytes() == bits(sort.oracle_sort(a, kt), kt).tobytes()
+
+
 def test_errors(ms):
     with pytest.raises(ms.MsortError):
         ms.msort_sort(0, 10, "u32", 1)
