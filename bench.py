@@ -549,7 +549,7 @@ def main():
     peaks = None
     if not args.no_links:
         try:
-            pk = ctx.measure_links(min(c * K, 4 << 30), 3)
+            pk = ctx.measure_links(min(c * K, 1 << 30), 3)  # (1 GiB per copy: 8 ranks x 2 pinned buffers stay small)
             if dist:  # the slowest rank's rates
                 for k in ("p2p_ce_gbs", "p2p_sm_gbs", "h2d_gbs", "d2h_gbs", "bidir_gbs"):
                     tt = torch.tensor([pk[k]], dtype=torch.float64)
