@@ -354,13 +354,14 @@ int radix_begin(msort_ctx* ctx, Rank& R, const void* src, uint64_t c) {
 
 // skewed-pass ranking (MSORT_SKEW_MODE, tuning only): 0 = peer match, 1 = one
 // atomic per warp row for each of the 4 most frequent digit values, 2 (default)
-// = 1 when one digit holds > 1/4 of the keys, else 0
+// = 1 when one digit holds > 1/4 of the keys, else 0; 3 = plain atomic ranking
+// (same-address lanes serialised) for every skewed pass
 int skew_mode() {
     static int v = -1;
     if (v < 0) {
         const char* e = std::getenv("MSORT_SKEW_MODE");
         v = e ? std::atoi(e) : 2;
-        if (v < 0 || v > 2) v = 2;
+        if (v < 0 || v > 3) v = 2;
     }
     return v;
 }
@@ -413,9 +414,9 @@ int radix_passes(msort_ctx* ctx, Rank& R, const void* src, void* dst, void* tmp,
         const uint64_t maxbin = ctx->skip_trivial ? uint64_t(R.h_trivial[8 + pid]) : 0;
         const bool skewed = maxbin * 16 > c;
         const int mode = skew_mode();
-        const bool dominant = mode == 1 ? skewed : (mode == 0 ? false : maxbin * 4 > c);
+        const bool dominant = mode == 1 ? skewed : (mode == 0 || mode == 3 ? false : maxbin * 4 > c);
         bool atomic_rank = j == 0 || atomic_rank_ok(R.st);
-        if (skewed && !dominant) atomic_rank = false;  // peer match
+        if (skewed && !dominant && mode != 3) atomic_rank = false;  // peer match
         const bool hot = dominant && atomic_rank;
         const int flags = (j == 0 ? 1 : 0) | (j == E - 1 ? 2 : 0) | (atomic_rank ? 4 : 0) | (hot ? 8 : 0);
         if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_pass[j][0], R.st));
