@@ -716,7 +716,9 @@ def main():
             "verified": verify["verified"], "verify_method": verify["method"],
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": main_run["launches"],
             "clocks": clk.summary(), "wall_s_timed_region": wall,
-            "step_ms": {"min": min(main_run["step_ms"]), "max": max(main_run["step_ms"])},
+            "step_ms": {"min": min(main_run["step_ms"]), "max": max(main_run["step_ms"]),
+                        "median": sorted(main_run["step_ms"])[len(main_run["step_ms"]) // 2],
+                        "mean_this_rank": sum(main_run["step_ms"]) / len(main_run["step_ms"])},
             "phases_ms": {"hist": main_run["hist_ms"] / args.steps,
                           "onesweep_passes": main_run["pass_ms"] / args.steps,
                           "merge_phase": merge_phase_ms},
