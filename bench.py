@@ -723,7 +723,7 @@ def main():
                           "onesweep_passes": main_run["pass_ms"] / args.steps,
                           "merge_phase": merge_phase_ms},
             "stages": {k: stage_info[k] for k in ("stage_label", "stage_pivot", "stage_max_x", "stage_ms",
-                                                  "stage_exchange_ms")} if stage_info and g > 1 else None,
+                                                  "stage_exchange_ms", "stage_pivot_ms")} if stage_info and g > 1 else None,
             "nvlink": nvlink, "links": peaks, "nccl_swap": nccl_leg,
             "paper_context": PAPER_CONTEXT,
             "het_baseline": het, "het_out_of_core": het_ooc,

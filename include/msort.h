@@ -182,6 +182,8 @@ typedef struct {
                                                            between distinct devices (or none needed)   */
     double   stage_swap_ms[MSORT_MAX_STAGES];           /* the transfer alone (modes 1 / 4: copy or NCCL
                                                            send/recv; fused modes: = stage_exchange_ms) */
+    double   stage_pivot_ms[MSORT_MAX_STAGES];          /* stage start .. exchange start: the pivot search
+                                                           (S4; modes 1 / 4 include its host read-back) */
 } msort_timings;
 
 int msort_get_timings(const msort_ctx* ctx, msort_timings* out);

@@ -63,6 +63,7 @@ class msort_timings(ctypes.Structure):
         ("stage_exchange_ms", ctypes.c_double * MSORT_MAX_STAGES),
         ("kernel_launches", ctypes.c_int), ("exchange_mode", ctypes.c_int), ("peer_bulk_ok", ctypes.c_int),
         ("stage_swap_ms", ctypes.c_double * MSORT_MAX_STAGES),
+        ("stage_pivot_ms", ctypes.c_double * MSORT_MAX_STAGES),
     ]
 
     def as_dict(self) -> dict:
@@ -80,6 +81,7 @@ class msort_timings(ctypes.Structure):
             "stage_exchange_ms": list(self.stage_exchange_ms[:S]),
             "kernel_launches": self.kernel_launches, "exchange_mode": self.exchange_mode,
             "peer_bulk_ok": self.peer_bulk_ok, "stage_swap_ms": list(self.stage_swap_ms[:S]),
+            "stage_pivot_ms": list(self.stage_pivot_ms[:S]),
         }
 
 

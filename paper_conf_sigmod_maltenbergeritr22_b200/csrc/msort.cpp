@@ -1550,16 +1550,18 @@ static void collect_exchange_timings(msort_ctx* ctx) {
     if (!ctx->timing) return;
     // e_xch events are recorded only on ranks that exchanged in that stage
     for (int s = 0; s < ctx->tm.n_stages; ++s) {
-        double mx = 0, sw = 0;
+        double mx = 0, sw = 0, pv = 0;
         for (int i = 0; i < ctx->nlocal; ++i) {
             Rank& R = ctx->r[i];
             if (!R.xch_rec[s]) continue;
             cudaSetDevice(R.dev);
             mx = std::max(mx, double(elapsed(R.e_xch[s][0], R.e_xch[s][1])));
+            pv = std::max(pv, double(elapsed(R.e_stage[s][0], R.e_xch[s][0])));
             if (ctx->xmode == 1 || ctx->xmode == 4)
                 sw = std::max(sw, double(elapsed(R.e_xch[s][0], R.e_swp[s])));
         }
         ctx->tm.stage_exchange_ms[s] = mx;
+        ctx->tm.stage_pivot_ms[s] = pv;
         // the transfer alone: separate in modes 1 / 4, the same as the exchange when fused (modes 0, 2)
         ctx->tm.stage_swap_ms[s] = (ctx->xmode == 1 || ctx->xmode == 4) ? sw : mx;
     }

@@ -279,6 +279,9 @@ def test_p2p_sort_virtual_ranks(ms, g, dist):
     for s, st in enumerate(stages):
         assert tm["stage_pivot"][s][: len(st)] == [op.p for op in st]
         assert tm["stage_max_x"][s] == max(max(op.xs) for op in st)
+    # per-stage timings: the pivot search is part of the stage, the exchange too
+    for pv, ex, st in zip(tm["stage_pivot_ms"], tm["stage_exchange_ms"], tm["stage_ms"]):
+        assert 0 < pv <= st and 0 <= ex <= st
 
 
 def _staged_chunks(ms, a, kt, g, exchange, stop):
