@@ -27,6 +27,8 @@
 #include <mutex>
 #include <string>
 #include <thread>
+
+#include <unistd.h>
 #include <tuple>
 #include <vector>
 
@@ -588,7 +590,16 @@ constexpr int kBounce = 3;
 class CopyPool {  // parallel memcpy on the host cores (persistent workers)
   public:
     static CopyPool& get() {
-        static CopyPool* p = new CopyPool;  // (never destroyed: its detached workers wait on it until exit)
+        // never destroyed (its detached workers wait on it until exit); a process forked after the
+        // pool started has no workers, so it builds its own
+        static std::mutex mu;
+        static CopyPool* p = nullptr;
+        static pid_t owner = 0;
+        std::lock_guard<std::mutex> lk(mu);
+        if (!p || owner != getpid()) {
+            p = new CopyPool;
+            owner = getpid();
+        }
         return *p;
     }
     void copy(void* dst, const void* src, size_t bytes) {
