@@ -603,3 +603,23 @@ def test_p2p_sort_distinct_gpus(ms, g, exchange):
         for s, st in enumerate(stages):
             assert tm["stage_pivot"][s][: len(st)] == [op.p for op in st]
     ctx.close()
+
+
+@pytest.mark.parametrize("exchange", [0, 1, 2, 4])
+def test_timing_off_every_mode(ms, exchange):
+    """MSORT_OPT_TIMING = 0 (no per-phase events) leaves every exchange mode's result and stage
+    statistics intact."""
+    g, c = 4, 3 * 7168 + 8
+    a = mi.np_generate(g * c, "u32", "reverse", seed=exchange + 50)
+    ctx = ms.Context(g, g * c, "u32", device_ids=[0] * g)
+    ctx.set_option(ms.MSORT_OPT_TIMING, 0)
+    ctx.set_option(ms.MSORT_OPT_EXCHANGE, exchange)
+    chunks = [dev_keys(a[i * c:(i + 1) * c]) for i in range(g)]
+    ctx.sort_device([ms.tensor_ptr(t) for t in chunks], c)
+    torch.cuda.synchronize()
+    out = np.concatenate([host_keys(t, "u32") for t in chunks])
+    tm = ctx.timings()
+    ctx.close()
+    assert np.array_equal(out, sort.oracle_sort(a, "u32"))
+    if exchange != 2:  # reverse input: every mirrored pair swaps whole chunks in every stage (x_d = c)
+        assert tm["stage_max_x"] == [c] * (g - 1)
