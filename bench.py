@@ -529,20 +529,24 @@ def main():
             if int(okt.item()) == 0:
                 nccl_leg = {"unavailable": err or "NCCL init failed on another rank"}
             else:
-                ctx.set_option(ms.MSORT_OPT_EXCHANGE, 4)
-                for _ in range(2):
-                    with torch.cuda.stream(stream):
-                        work.copy_(pristine)
-                    sort_dev()
-                barrier()
-                r4 = timed_steps(args.steps)
-                v4 = verify_all(verify_local(work, pristine, valid, kt), dist)
-                t4 = r4["tm"]
-                st4 = {"stage_label": t4["stage_label"], "stage_max_x": t4["stage_max_x"],
-                       "stage_exchange_ms": [max_over_ranks(x) for x in t4["stage_swap_ms"]]}
-                nccl_leg = {"value": n / (r4["ms_per_step"] / 1e3), "unit": "keys/s", "ms_per_step": r4["ms_per_step"],
-                            "exchange": "Alg.2, swap as grouped ncclSend/ncclRecv per mirrored pair, then local merge",
-                            "verified": v4["verified"], "swap_stage_ms": st4["stage_exchange_ms"], "stages": st4}
+                try:  # (a failure here must not cost the headline line printed below)
+                    ctx.set_option(ms.MSORT_OPT_EXCHANGE, 4)
+                    for _ in range(2):
+                        with torch.cuda.stream(stream):
+                            work.copy_(pristine)
+                        sort_dev()
+                    barrier()
+                    r4 = timed_steps(args.steps)
+                    v4 = verify_all(verify_local(work, pristine, valid, kt), dist)
+                    t4 = r4["tm"]
+                    st4 = {"stage_label": t4["stage_label"], "stage_max_x": t4["stage_max_x"],
+                           "stage_exchange_ms": [max_over_ranks(x) for x in t4["stage_swap_ms"]]}
+                    nccl_leg = {"value": n / (r4["ms_per_step"] / 1e3), "unit": "keys/s",
+                                "ms_per_step": r4["ms_per_step"],
+                                "exchange": "Alg.2, swap as grouped ncclSend/ncclRecv per mirrored pair, then local merge",
+                                "verified": v4["verified"], "swap_stage_ms": st4["stage_exchange_ms"], "stages": st4}
+                except Exception as e:
+                    nccl_leg = {"failed": str(e)[:500]}
             ctx.set_option(ms.MSORT_OPT_EXCHANGE, args.exchange)
 
     # --- interconnect peaks (msort_measure_links; every rank, collective in dist mode)
