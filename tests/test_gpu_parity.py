@@ -131,6 +131,28 @@ def test_step_histogram(ms, kt):
     assert np.array_equal(got.astype(np.uint64), radix.histograms(a, kt))
 
 
+@pytest.mark.parametrize("kt", ["u64", "f64"])
+def test_step_histogram_8byte_skewed_large(ms, kt):
+    """4e8 8-byte keys (~2600 per thread of 148 x 1024, so every private counter column sees thousands of
+    adds), all but 1 in 997 on ONE bin per pass, read from one key past a 16-byte boundary (head and tail
+    keys).  Expected: the oracle's histogram of the random keys plus the constant key's bins times its
+    count (closed form)."""
+    n = 400_000_003
+    const = np.array([0x40091EB851EB851F], dtype=np.uint64)  # (as f64: 3.14; codec T applied by the oracle)
+    d = torch.full((n,), int(const.view(np.int64)[0]), dtype=torch.int64, device="cuda")
+    idx = torch.arange(1, n, 997, device="cuda")
+    rnd = mi.np_generate(len(idx), kt, "uniform", seed=11)
+    d[idx] = torch.from_numpy(rnd.view(np.int64).copy()).cuda()
+    P = radix.num_passes(kt)
+    h = torch.zeros(P * 256, dtype=torch.int32, device="cuda")
+    ms.msort_step_histogram(ms.tensor_ptr(d) + 8, n - 1, kt, ms.tensor_ptr(h))  # keys d[1:]
+    torch.cuda.synchronize()
+    got = h.cpu().numpy().view(np.uint32).reshape(P, 256).astype(np.uint64)
+    n_const = (n - 1) - len(idx)
+    want = radix.histograms(rnd.view(mi.NP_DTYPE[kt]), kt) + radix.histograms(const.view(mi.NP_DTYPE[kt]), kt) * n_const
+    assert np.array_equal(got, want)
+
+
 @pytest.mark.parametrize("kt", ["u32", "u64", "f32"])
 def test_step_radix_pass(ms, kt):
     n = 50001
