@@ -228,7 +228,10 @@ struct OsCfg {
 // may override single parameters with -DMSORT_W32=4 etc.):
 //   u32/f32: 7168-key tiles, 4 blocks of 256 threads per SM, look-back window 2,
 //            groups of 32, next tile counted after the scatter (3 barriers)
-//   u64/f64: 3584-key tiles, 4 blocks per SM, window 1, groups of 16
+//   u64/f64: 7680-key tiles, 2 blocks of 512 threads per SM, window 2, groups
+//            of 16, next tile counted after the scatter (session 3: 7.78 ms per
+//            2e9-key u64 pass vs 8.35 for 3584-key tiles of 256 threads, window
+//            1, four barriers; profiles/radix_tuning_r2.md)
 #ifndef MSORT_T32
 #define MSORT_T32 256
 #endif
@@ -245,7 +248,7 @@ struct OsCfg {
 #define MSORT_G32 32
 #endif
 #ifndef MSORT_W64
-#define MSORT_W64 1  // round 2: 8.24 ms per 2e9-key u64 pass vs 8.45 at window 4 (profiles/radix_tuning_r2.md)
+#define MSORT_W64 2
 #endif
 #ifndef MSORT_G64
 #define MSORT_G64 16
@@ -255,9 +258,18 @@ struct OsCfg {
 #endif
 #define MSORT_CFG32 OsCfg<MSORT_T32, MSORT_I32, 0x5555555u, MSORT_B32, MSORT_W32, MSORT_G32, true>
 #ifndef MSORT_CE64
-#define MSORT_CE64 false  // (counting the next tile after the scatter: 3% slower for 8-byte keys in round 1)
+#define MSORT_CE64 true
 #endif
-#define MSORT_CFG64 OsCfg<256, 14, 0x1555u, 4, MSORT_W64, MSORT_G64, MSORT_CE64>
+#ifndef MSORT_T64
+#define MSORT_T64 512
+#endif
+#ifndef MSORT_I64
+#define MSORT_I64 15
+#endif
+#ifndef MSORT_B64
+#define MSORT_B64 2
+#endif
+#define MSORT_CFG64 OsCfg<MSORT_T64, MSORT_I64, 0x1555u, MSORT_B64, MSORT_W64, MSORT_G64, MSORT_CE64>
 using Cfg32 = MSORT_CFG32;
 using Cfg64 = MSORT_CFG64;
 template <typename U>
