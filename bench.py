@@ -379,6 +379,21 @@ def nvlink_fractions(stages: dict, K: int, peaks: dict | None, same_device: bool
                      "distinct GPUs: NVLink 5 through NVSwitch")}
 
 
+def baseline_config_name(n: int, kt: str, dist: str) -> str:
+    """Which BASELINE.json config a bench run measures (the N=1 headline is configs[2])."""
+    if n == 4_000_000_000 and kt == "u32" and dist == "uniform":
+        return "BASELINE.json configs[2], paper Fig.1 shape"
+    if n == 2_000_000_000 and kt == "u32" and dist != "uniform":
+        return "BASELINE.json configs[3] key distribution"
+    if n == 2_000_000_000 and kt in ("u64", "f32"):
+        return "BASELINE.json configs[4] key type"
+    if n == 1 << 28 and kt == "u32":
+        return "BASELINE.json configs[1] size"
+    if n == 1 << 20 and kt == "u32":
+        return "BASELINE.json configs[0] size"
+    return "not a BASELINE.json configuration"
+
+
 def main():
     args = parse()
     args.n = int(args.n)
@@ -714,7 +729,7 @@ def main():
             "metric": "keys/sec", "value": value, "unit": "keys/s", "n_gpus": g, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": kt, "data": "synthetic",
-            "config": {"workload": f"{n} {args.dist} {kt} keys (BASELINE.json configs[2], paper Fig.1 shape), "
+            "config": {"workload": f"{n} {args.dist} {kt} keys ({baseline_config_name(n, kt, args.dist)}), "
                                    f"device-resident P2P sort on {g} GPU(s)",
                        "n": n, "keys_per_gpu": c, "key_type": kt, "distribution": args.dist, "seed": args.seed,
                        "parallelism": f"p2p{g}", "l2": "inputs 16 GB >> 126 MB L2 (no flush needed)",
