@@ -4,7 +4,7 @@ non-decreasing under T, a permutation of the input (multiset fingerprint), and
 sampled outputs equal to the oracle's order statistics computed one by one.
 Together these imply byte equality with the (unique) oracle result.
 
-configs[2]: 4e9 uniform u32 on one GPU (the bench's N=1 workload);
+configs[2]: 4e9 uniform u32 on one GPU (the bench's N=1 workload); configs[4]'s u64 / f32 at 2e9 on one GPU;
 configs[1]: 2^28 uniform u32 on 2 chunks (virtual ranks on one GPU);
 configs[3]/[4]: 2e9 keys on 8 chunks (virtual ranks): zipf / reverse / nearly-sorted / sorted / normal
 u32, f32, u64, NEXT-1 on zipf, and the NCCL swap (mode 4) on reverse.
@@ -106,6 +106,20 @@ def test_config3_4e9_u32_one_gpu():
     torch.cuda.synchronize()
     ctx.close()
     _check(chunks, n, "u32", "uniform", 1)
+
+
+@pytest.mark.parametrize("kt", ["u64", "f32"])
+def test_config4_2e9_one_gpu(kt):
+    """configs[4]'s key types as bench.py times them at N = 1 (2e9 keys in one chunk: 8-byte keys with the
+    7680-key tiles of 512 threads, float keys with the codec fused into the first / last pass)."""
+    import paper_conf_sigmod_maltenbergeritr22_b200 as ms
+    n = 2_000_000_000
+    chunks, c = _gen_chunks(n, 1, kt, "uniform", 5)
+    ctx = ms.Context(1, n, kt, device_ids=[0])
+    ctx.sort_device([ms.tensor_ptr(chunks[0])], c)
+    torch.cuda.synchronize()
+    ctx.close()
+    _check(chunks, n, kt, "uniform", 5)
 
 
 def test_max_chunk_u32_one_gpu():
