@@ -31,6 +31,16 @@ namespace {
 // ---------------------------------------------------------------------------
 // S2: digit histograms of T(key) for every pass, one read of the chunk.
 // ---------------------------------------------------------------------------
+// Cache operators of the onesweep pass's tile loads and scatter stores (build
+// parameters).  ld.global.cg keeps the streamed keys out of L1: no L1 fill in
+// the data pipe that binds the pass (session 3: 2e9-key u64 pass 7.71 -> 7.13
+// ms, u32 / f32 about 1 % faster than ld.global.cs; profiles/radix_tuning_r2.md)
+#ifndef MSORT_TILE_LD
+#define MSORT_TILE_LD __ldcg
+#endif
+#ifndef MSORT_TILE_ST
+#define MSORT_TILE_ST __stcs
+#endif
 constexpr int kHistThreads = 1024;
 constexpr int kHistUnroll = 4;
 
@@ -323,7 +333,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
         const U* src = in + tb + wofs;
         if (tb + TILE <= n) {
 #pragma unroll
-            for (int i = 0; i < ITEMS; ++i) keys[i] = __ldcs(src + i * 32);
+            for (int i = 0; i < ITEMS; ++i) keys[i] = MSORT_TILE_LD(src + i * 32);
         } else {
 #pragma unroll
             for (int i = 0; i < ITEMS; ++i) {
@@ -567,7 +577,7 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
             for (int i = 0; i < ITEMS; ++i) {
                 const uint32_t j = tid + i * THREADS;
                 const U k = s_keys[j];
-                __stcs(out + s_delta[uint32_t(k >> shift) & 0xFF] + j, DEC_OUT ? decode<U, FLOAT>(k) : k);
+                MSORT_TILE_ST(out + s_delta[uint32_t(k >> shift) & 0xFF] + j, DEC_OUT ? decode<U, FLOAT>(k) : k);
             }
         } else {
             const uint32_t valid = uint32_t(n - tile_base);
