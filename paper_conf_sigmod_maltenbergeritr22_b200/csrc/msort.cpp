@@ -682,7 +682,9 @@ int bounce_h2d(Rank& R, void* dst, const char* src, size_t bytes, cudaStream_t s
     for (size_t off = 0, k = 0; off < bytes; off += kBounceBytes, ++k) {
         const int b = int(k % kBounce);
         const size_t len = std::min(kBounceBytes, bytes - off);
-        if (k >= size_t(kBounce)) CUDA_TRY(cudaEventSynchronize(R.e_bounce[b]));  // its last DMA is done
+        // its last DMA is done (also one queued by an earlier call: the pipelined path stages piece by piece;
+        // an event never recorded counts as complete)
+        CUDA_TRY(cudaEventSynchronize(R.e_bounce[b]));
         CopyPool::get().copy(R.bounce[b], src + off, len);
         CUDA_TRY(cudaMemcpyAsync(d + off, R.bounce[b], len, cudaMemcpyHostToDevice, st));
         CUDA_TRY(cudaEventRecord(R.e_bounce[b], st));
@@ -1630,7 +1632,7 @@ static constexpr uint64_t kPipeMinKeys = 1ull << 20;
 // 0+1 and 2+3 merged into B0.  Leaves two sorted runs: B0[0, *split) and
 // B0[*split, c).  Records e_h2d0/e_h2d1 (copy stream), e_begin/e_sorted/e_merged.
 static int load_sort_pieces(msort_ctx* ctx, Rank& R, const char* host, uint64_t n, uint64_t c, char* dst_stage,
-                            uint64_t* split) {
+                            uint64_t* split, bool pageable = false) {
     const size_t K = key_bytes(ctx->kt);
     char* stage = dst_stage;
     char* b0 = static_cast<char*>(R.buf[0]);
@@ -1641,16 +1643,24 @@ static int load_sort_pieces(msort_ctx* ctx, Rank& R, const char* host, uint64_t 
     CUDA_TRY(cudaEventRecord(R.e_merged, R.st));
     CUDA_TRY(cudaStreamWaitEvent(R.cst, R.e_merged, 0));
     CUDA_TRY(cudaEventRecord(R.e_h2d0, R.cst));
-    for (int i = 0; i < kPieces; ++i) {
+    auto h2d_piece = [&](int i) -> int {
         const uint64_t lo = std::min(pb[i], n), hi = std::min(pb[i + 1], n);
-        if (hi > lo) CUDA_TRY(cudaMemcpyAsync(stage + lo * K, host + lo * K, (hi - lo) * K, cudaMemcpyHostToDevice, R.cst));
+        if (hi > lo) {
+            if (pageable)  // (returns once the host threads have staged the whole piece)
+                MSORT_TRY(bounce_h2d(R, stage + lo * K, host + lo * K, (hi - lo) * K, R.cst));
+            else
+                CUDA_TRY(cudaMemcpyAsync(stage + lo * K, host + lo * K, (hi - lo) * K, cudaMemcpyHostToDevice, R.cst));
+        }
         if (i == kPieces - 1 && c > n) {
             CUDA_TRY(launch_fill_max(stage + n * K, c - n, ctx->kt, R.cst));
             ctx->tm.kernel_launches += 1;
         }
         CUDA_TRY(cudaEventRecord(R.e_piece[i], R.cst));
-    }
-    CUDA_TRY(cudaEventRecord(R.e_h2d1, R.cst));
+        if (i == kPieces - 1) CUDA_TRY(cudaEventRecord(R.e_h2d1, R.cst));
+        return MSORT_OK;
+    };
+    // pinned: every copy queued at once; pageable: the host stages piece i+1 while the GPU sorts piece i
+    for (int i = 0; i < (pageable ? 1 : kPieces); ++i) MSORT_TRY(h2d_piece(i));
     // S1-S3 per piece on the compute stream, round-1 merges as soon as possible
     CUDA_TRY(cudaEventRecord(R.e_begin, R.st));
     for (int i = 0; i < kPieces; ++i) {
@@ -1666,13 +1676,14 @@ static int load_sort_pieces(msort_ctx* ctx, Rank& R, const char* host, uint64_t 
                                   &ctx->tm.kernel_launches));
         }
         if (i == kPieces - 1) CUDA_TRY(cudaEventRecord(R.e_sorted, R.st));
+        if (pageable && i + 1 < kPieces) MSORT_TRY(h2d_piece(i + 1));
     }
     CUDA_TRY(cudaEventRecord(R.e_merged, R.st));
     *split = pb[2];
     return MSORT_OK;
 }
 
-static int sort_host_pipelined(msort_ctx* ctx, char* host, uint64_t n, uint64_t c) {
+static int sort_host_pipelined(msort_ctx* ctx, char* host, uint64_t n, uint64_t c, bool pageable) {
     Rank& R = ctx->r[0];
     const size_t K = key_bytes(ctx->kt);
     CUDA_TRY(cudaSetDevice(R.dev));
@@ -1680,7 +1691,7 @@ static int sort_host_pipelined(msort_ctx* ctx, char* host, uint64_t n, uint64_t 
     char* stage = static_cast<char*>(R.stage);
     char* b0 = static_cast<char*>(R.buf[0]);
     uint64_t split = 0;
-    MSORT_TRY(load_sort_pieces(ctx, R, host, n, c, stage, &split));
+    MSORT_TRY(load_sort_pieces(ctx, R, host, n, c, stage, &split, pageable));
     // S8 overlapped with the final merge: slice co-ranks, then merge + D2H per slice
     const char* A = b0;
     const uint64_t al = split;
@@ -1698,19 +1709,32 @@ static int sort_host_pipelined(msort_ctx* ctx, char* host, uint64_t n, uint64_t 
     int ends[kSlices], ns = 0;
     for (int e : {1, 4, 16, nsteps})
         if (e <= nsteps && (ns == 0 || e > ends[ns - 1])) ends[ns++] = e;
+    auto slice_lo = [&](int s) { return uint64_t(s ? ends[s - 1] : 0) * step; };
+    auto slice_hi = [&](int s) { return std::min(c, uint64_t(ends[s]) * step); };
+    auto d2h_slice = [&](int s) -> int {
+        const uint64_t lo = slice_lo(s), dhi = std::min(slice_hi(s), n);
+        CUDA_TRY(cudaStreamWaitEvent(R.cst, R.e_slice[s], 0));
+        if (s == 0) CUDA_TRY(cudaEventRecord(R.e_d2h0, R.cst));
+        if (dhi > lo) {
+            if (pageable)  // (returns once the slice is in host memory; later slices keep merging meanwhile)
+                MSORT_TRY(bounce_d2h(R, host + lo * K, stage + lo * K, (dhi - lo) * K, R.cst));
+            else
+                CUDA_TRY(cudaMemcpyAsync(host + lo * K, stage + lo * K, (dhi - lo) * K, cudaMemcpyDeviceToHost, R.cst));
+        }
+        return MSORT_OK;
+    };
     for (int s = 0; s < ns; ++s) {
         const int j0 = s ? ends[s - 1] : 0, j1 = ends[s];
-        const uint64_t lo = uint64_t(j0) * step, hi = std::min(c, uint64_t(j1) * step);
+        const uint64_t lo = slice_lo(s), hi = slice_hi(s);
         const uint64_t a0 = R.h_pivot[j0], a1 = R.h_pivot[j1];
         const uint64_t b0i = lo - a0, b1i = hi - a1;
         CUDA_TRY(launch_merge(A + a0 * K, a1 - a0, B + b0i * K, b1i - b0i, stage + lo * K, ctx->kt, R.mws, R.st,
                               &ctx->tm.kernel_launches));
         CUDA_TRY(cudaEventRecord(R.e_slice[s], R.st));
-        CUDA_TRY(cudaStreamWaitEvent(R.cst, R.e_slice[s], 0));
-        if (s == 0) CUDA_TRY(cudaEventRecord(R.e_d2h0, R.cst));
-        const uint64_t dhi = std::min(hi, n);
-        if (dhi > lo) CUDA_TRY(cudaMemcpyAsync(host + lo * K, stage + lo * K, (dhi - lo) * K, cudaMemcpyDeviceToHost, R.cst));
+        if (!pageable) MSORT_TRY(d2h_slice(s));
     }
+    if (pageable)
+        for (int s = 0; s < ns; ++s) MSORT_TRY(d2h_slice(s));
     CUDA_TRY(cudaEventRecord(R.e_end, R.st));
     CUDA_TRY(cudaEventRecord(R.e_d2h1, R.cst));
     CUDA_TRY(cudaEventSynchronize(R.e_d2h1));
@@ -1740,9 +1764,9 @@ int msort_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n) {
     reset_timings(ctx, c);
     const size_t K = key_bytes(ctx->kt);
     char* host = static_cast<char*>(host_keys);
-    // pageable keys: through pinned bounce buffers (no transfer/sort overlap, but PCIe rate)
+    // pageable keys: through pinned bounce buffers (one GPU: pipelined like pinned keys, piece by piece)
     const bool pageable = host_is_pageable(host_keys);
-    if (g == 1 && ctx->host_pipeline && c >= kPipeMinKeys && !pageable) return sort_host_pipelined(ctx, host, n, c);
+    if (g == 1 && ctx->host_pipeline && c >= kPipeMinKeys) return sort_host_pipelined(ctx, host, n, c, pageable);
     for (int i = 0; i < g; ++i) {
         Rank& R = ctx->r[i];
         CUDA_TRY(cudaSetDevice(R.dev));

@@ -470,11 +470,13 @@ def test_msort_sort_host_pointer(ms, n, kt):
     assert bits(h, kt).tobytes() == bits(sort.oracle_sort(a, kt), kt).tobytes()
 
 
-@pytest.mark.parametrize("n,kt,g", [(50_000_003, "u32", 1), (20_000_001, "f64", 2), (33_554_437, "u64", 4)])
+@pytest.mark.parametrize("n,kt,g", [(50_000_003, "u32", 1), (20_000_001, "f64", 2), (33_554_437, "u64", 4),
+                                    (300_000_001, "u32", 1), (100_000_003, "u64", 1)])
 def test_pageable_host_bounce(ms, n, kt, g):
     """Pageable host keys (numpy) spanning several 64 MiB pinned bounce buffers: the host threads' copies,
     the bounce ring's events and the padding of the last chunk, through msort_sort (the north-star entry,
-    g = 1) and a context (virtual ranks)."""
+    g = 1: the pipelined path, the host staging piece i+1 while the GPU sorts piece i, each piece and each
+    D2H slice several bounce buffers long) and a context (virtual ranks)."""
     a = mi.np_generate(n, kt, "uniform", seed=n % 97)
     h = a.copy()
     if g == 1:
