@@ -2012,7 +2012,7 @@ static int dist_barrier(msort_ctx* ctx) {
 
 // c = chunk keys, valid = real keys in it (the rest is padded here, reading Q3)
 static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream, bool keep_timings,
-                          const char* host, uint64_t valid);
+                          const char* host, uint64_t valid, bool pageable = false);
 
 int msort_plan_chunk(uint64_t n, int g, int rank, uint64_t* c, uint64_t* offset, uint64_t* valid) {
     if (!valid_g(g) || rank < 0 || rank >= g) return set_error(MSORT_ERR_INVALID_ARGUMENT, "bad g or rank");
@@ -2198,9 +2198,10 @@ int msort_dist_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n_total) {
     reset_timings(ctx, c);
     const size_t K = key_bytes(ctx->kt);
     const bool pageable = valid && host_is_pageable(host_keys);
-    if (ctx->host_pipeline && c >= kPipeMinKeys && !pageable) {
-        // pipelined S0 (MSORT_OPT_HOST_PIPELINE): H2D pieces sorted as they land (the pad is filled there)
-        MSORT_TRY(dist_sort_impl(ctx, R.stage, c, R.st, true, static_cast<const char*>(host_keys), valid));
+    if (ctx->host_pipeline && c >= kPipeMinKeys) {
+        // pipelined S0 (MSORT_OPT_HOST_PIPELINE): H2D pieces sorted as they land (the pad is filled there);
+        // pageable keys: the host stages piece i+1 through the bounce buffers while the GPU sorts piece i
+        MSORT_TRY(dist_sort_impl(ctx, R.stage, c, R.st, true, static_cast<const char*>(host_keys), valid, pageable));
     } else {
         CUDA_TRY(cudaEventRecord(R.e_h2d0, R.st));
         if (pageable) MSORT_TRY(bounce_h2d(R, R.stage, static_cast<const char*>(host_keys), valid * K, R.st));
@@ -2220,7 +2221,7 @@ int msort_dist_sort_host(msort_ctx* ctx, void* host_keys, uint64_t n_total) {
 }
 
 static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* stream, bool keep_timings,
-                          const char* host, uint64_t valid) {
+                          const char* host, uint64_t valid, bool pageable) {
     if (!ctx || !ctx->dist || !ctx->imported) return set_error(MSORT_ERR_INVALID_ARGUMENT, "dist ctx not imported");
     if (c && !d_chunk) return set_error(MSORT_ERR_INVALID_ARGUMENT, "NULL chunk");
     MSORT_TRY(check_c(ctx, c));
@@ -2242,7 +2243,7 @@ static int dist_sort_impl(msort_ctx* ctx, void* d_chunk, uint64_t c, void* strea
     void* sorted_dst = g == 1 ? d_chunk : R.buf[1];
     if (host) {
         uint64_t split = 0;
-        MSORT_TRY(load_sort_pieces(ctx, R, host, valid, c, static_cast<char*>(d_chunk), &split));
+        MSORT_TRY(load_sort_pieces(ctx, R, host, valid, c, static_cast<char*>(d_chunk), &split, pageable));
         const char* b0 = static_cast<const char*>(R.buf[0]);
         CUDA_TRY(launch_merge(b0, split, b0 + split * key_bytes(ctx->kt), c - split, sorted_dst, ctx->kt, R.mws, R.st,
                               &ctx->tm.kernel_launches));

@@ -51,7 +51,11 @@ def _worker(rank, world, port, n, kt, distn, out_dir, host, exchange=0, nccl=Fal
     ctx.set_option(m.MSORT_OPT_EXCHANGE, exchange)
     a = mi.np_generate(n, kt, distn, seed=5)
     mine = codec.bits_of(a[off:off + v], kt).copy()   # this rank's slice; the library pads (reading Q3)
-    if host:
+    if host == "pageable":  # a plain numpy array: the bounce-buffer path
+        h = mine.view(np.uint8).copy()
+        ctx.sort_host(h.ctypes.data, n)
+        res = h
+    elif host:
         h = torch.from_numpy(mine.view(np.uint8).copy()).pin_memory()
         ctx.sort_host(m.tensor_ptr(h), n)
         res = h.numpy()
@@ -84,6 +88,9 @@ def _worker(rank, world, port, n, kt, distn, out_dir, host, exchange=0, nccl=Fal
     (2, 2_500_001, "u32", "uniform", True, 0),
     (4, 4_400_000, "f32", "uniform", True, 2),
     (2, 2_200_002, "u32", "zipf", True, 3),
+    # pageable host keys: bounce buffers, below and above the pipelining threshold
+    (2, 60_001, "u64", "uniform", "pageable", 0),
+    (2, 2_500_001, "u32", "uniform", "pageable", 0),
 ])
 def test_dist_sort_matches_oracle(tmp_path, world, n, kt, distn, host, exchange):
     mp.spawn(_worker, args=(world, _free_port(), n, kt, distn, str(tmp_path), host, exchange), nprocs=world,
