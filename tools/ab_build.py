@@ -10,7 +10,7 @@ from paper_conf_sigmod_maltenbergeritr22_b200 import build as b  # noqa: E402
 
 rev = sys.argv[1] if len(sys.argv) > 1 else "HEAD"
 name = sys.argv[2] if len(sys.argv) > 2 else "base"
-defines = [a for a in sys.argv[3:] if a.startswith("-D")]
+defines = [a for a in sys.argv[3:] if a.startswith(("-D", "-X"))]  # defines and -Xptxas options
 dst = os.path.join(ROOT, "tools", "_ablate", name, "paper_conf_sigmod_maltenbergeritr22_b200")
 os.makedirs(os.path.join(dst, "_build"), exist_ok=True)
 tmp = tempfile.mkdtemp()
