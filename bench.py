@@ -602,6 +602,12 @@ def main():
                                  "pct_of_peak": pj.get("smem_wavefronts_pct_of_peak_sustained_elapsed"),
                                  "bank_conflicts_per_launch": pj.get("smem_bank_conflicts_per_launch"),
                                  "source": os.path.relpath(prof, ROOT) + " (ncu --set full capture)"}
+                    if pj.get("l1_pipe_wavefronts_per_32_keys"):
+                        # the pass's binding resource: the SM's L1 data pipe (shared + global wavefronts)
+                        smem_pipe["l1_data_pipe"] = {
+                            "wavefronts_per_32_keys": pj["l1_pipe_wavefronts_per_32_keys"],
+                            "global_wavefronts_per_32_keys": pj.get("l1_pipe_global_wavefronts_per_32_keys"),
+                            "pct_busy": pj.get("l1_pipe_pct_of_peak_sustained_elapsed")}
         except Exception:
             traffic = None
     P = K  # passes (8-bit digits)

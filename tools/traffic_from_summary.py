@@ -13,5 +13,14 @@ j = {"source": note, "keys_per_launch": int(n), "dram_bytes_read": rd, "dram_byt
      "smem_wavefronts_pct_of_peak_sustained_elapsed": g("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed"),
      "smem_bank_conflicts_per_launch": g("l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum"),
      "gpu_time_ms_cold": g("gpu__time_duration.sum")}
+try:  # the whole L1 data pipe (shared + global/local wavefronts), when the summary carries it
+    sms = g("device__attribute_multiprocessor_count")
+    sh = g("SM_A.TriageCompute.l1tex__data_pipe_lsu_wavefronts_mem_shared.avg") * sms
+    lg = g("SM_A.TriageCompute.l1tex__data_pipe_lsu_wavefronts_mem_lgds.avg") * sms
+    j["l1_pipe_wavefronts_per_32_keys"] = round((sh + lg) / (n / 32), 2)
+    j["l1_pipe_global_wavefronts_per_32_keys"] = round(lg / (n / 32), 2)
+    j["l1_pipe_pct_of_peak_sustained_elapsed"] = g("l1tex__data_pipe_lsu_wavefronts.sum.pct_of_peak_sustained_elapsed")
+except AttributeError:
+    pass
 json.dump(j, open(out, "w"), indent=1)
 print(out, round(j["dram_bytes_per_launch"] / j["algorithmic_bytes_per_launch"], 4), j["smem_wavefronts_per_32_keys"], j["gpu_time_ms_cold"])
