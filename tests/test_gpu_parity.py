@@ -101,6 +101,26 @@ def test_radix_sort_distributions(ms, dist):
     assert np.array_equal(host_keys(d, "u32"), sort.oracle_sort(a, "u32"))
 
 
+@pytest.mark.parametrize("shape", ["small_ints", "high_word", "few_doubles"])
+def test_radix_sort_skewed_8byte(ms, shape):
+    """Skewed 8-byte keys through the 512-thread u64/f64 tiles: every skew path of the pass (trivial passes
+    skipped, a dominant digit ranked by the hot path, moderately skewed digits by peer match), over several
+    7680-key tiles and a ragged one."""
+    n = 5 * 7680 + 3 * (1 << 16) + 11
+    z = mi.np_generate(n, "u32", "zipf_rank", seed=21).astype(np.uint64)
+    if shape == "small_ints":      # high bytes zero (trivial passes), bytes 1-2 dominated by one value
+        a, kt = z, "u64"
+    elif shape == "high_word":     # the skew sits in the upper passes, the low word is uniform
+        a, kt = (z << np.uint64(32)) | mi.np_generate(n, "u32", "uniform", seed=22).astype(np.uint64), "u64"
+    else:                          # 40 distinct doubles, zipf-weighted, with -0.0 / +0.0 among them
+        vals = np.concatenate([np.array([-0.0, 0.0]), np.linspace(-1e3, 1e3, 38)])
+        a, kt = vals[(z % np.uint64(40)).astype(np.int64)], "f64"
+    d = dev_keys(a)
+    ms.msort_sort(ms.tensor_ptr(d), n, kt, 1)
+    torch.cuda.synchronize()
+    assert np.array_equal(bits(host_keys(d, kt), kt), bits(sort.oracle_sort(a, kt), kt))
+
+
 def test_radix_sort_constant_and_special(ms):
     # all-equal keys (every pass trivial) and the IEEE special-value table
     for a, kt in [(np.full(50000, 7, np.uint32), "u32"), (np.full(9999, 0x7FC00000, np.uint32).view(np.float32), "f32")]:
