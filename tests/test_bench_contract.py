@@ -85,3 +85,18 @@ def test_output_verification_helpers():
         y = s.copy()
         y[-1] = y[-2]                                           # sorted, but not a permutation
         assert not b.verify_all(b.verify_local(torch.from_numpy(y), inp, len(a), kt, block=1024), None)["verified"], kt
+
+
+def test_workload_names_the_baseline_config():
+    """bench.py's `config.workload` names the BASELINE.json config it measures (the N=1 headline is configs[2])."""
+    import importlib.util
+    spec = importlib.util.spec_from_file_location("_bench", os.path.join(ROOT, "bench.py"))
+    b = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(b)
+    assert "configs[2]" in b.baseline_config_name(4_000_000_000, "u32", "uniform")
+    assert "configs[4]" in b.baseline_config_name(2_000_000_000, "u64", "uniform")
+    assert "configs[4]" in b.baseline_config_name(2_000_000_000, "f32", "uniform")
+    assert "configs[3]" in b.baseline_config_name(2_000_000_000, "u32", "zipf")
+    assert "configs[1]" in b.baseline_config_name(1 << 28, "u32", "uniform")
+    assert "configs[0]" in b.baseline_config_name(1 << 20, "u32", "uniform")
+    assert "not a BASELINE" in b.baseline_config_name(12345, "u32", "uniform")
