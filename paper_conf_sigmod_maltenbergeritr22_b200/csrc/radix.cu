@@ -266,7 +266,10 @@ struct OsCfg {
 #ifndef MSORT_LB_SLEEP_NS
 #define MSORT_LB_SLEEP_NS 32  // back-off of a look-back poll on an unpublished predecessor
 #endif
-#define MSORT_CFG32 OsCfg<MSORT_T32, MSORT_I32, 0x5555555u, MSORT_B32, MSORT_W32, MSORT_G32, true>
+#ifndef MSORT_BM32
+#define MSORT_BM32 0x7777777u  // peer-match ranking: items ranked by the ballot match (bit set; 3 of 4) vs smem atomicOr masks
+#endif
+#define MSORT_CFG32 OsCfg<MSORT_T32, MSORT_I32, MSORT_BM32, MSORT_B32, MSORT_W32, MSORT_G32, true>
 #ifndef MSORT_CE64
 #define MSORT_CE64 true
 #endif
