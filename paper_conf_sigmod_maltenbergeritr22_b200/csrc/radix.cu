@@ -282,7 +282,10 @@ struct OsCfg {
 #ifndef MSORT_B64
 #define MSORT_B64 2
 #endif
-#define MSORT_CFG64 OsCfg<MSORT_T64, MSORT_I64, 0x1555u, MSORT_B64, MSORT_W64, MSORT_G64, MSORT_CE64>
+#ifndef MSORT_BM64
+#define MSORT_BM64 0x1555u
+#endif
+#define MSORT_CFG64 OsCfg<MSORT_T64, MSORT_I64, MSORT_BM64, MSORT_B64, MSORT_W64, MSORT_G64, MSORT_CE64>
 using Cfg32 = MSORT_CFG32;
 using Cfg64 = MSORT_CFG64;
 template <typename U>
