@@ -37,6 +37,9 @@ RadixWs radix_ws_layout(void* ws, uint64_t n, int kt);
 // set trivial flags.  keys are raw (T applied on load).
 cudaError_t radix_prologue(const void* keys, uint64_t n, int kt, const RadixWs& ws, cudaStream_t st);
 // histogram only into an external [P][256] array (zeroed inside)
+// scan_kernel's per-pass outputs (RadixWs::trivial): [0,8) trivial pass, [8,16)
+// largest bin, [16,24) the 4 most frequent digit values, [24,32) keys on them
+constexpr int kTrivialWords = 32;
 cudaError_t launch_histogram(const void* keys, uint64_t n, int kt, uint32_t* hist, cudaStream_t st);
 // bases from hist rows (all P)
 cudaError_t launch_scan(const uint32_t* hist, uint32_t* base, uint32_t* trivial, uint64_t n, int kt, cudaStream_t st);

@@ -145,7 +145,7 @@ struct Rank {
     size_t mws_bytes = 0;
     uint64_t* d_pivot = nullptr;   // [128] pivots (Alg.2) or splitters (all-to-all)
     uint64_t* h_pivot = nullptr;   // pinned [128]
-    uint32_t* h_trivial = nullptr; // pinned [24]: trivial flags, largest bin per pass, its digit
+    uint32_t* h_trivial = nullptr; // pinned [kTrivialWords]: trivial flags, largest bin, hot digits per pass
     DevStage* d_stage = nullptr;   // device-resident Alg.2 state (exchange mode 0): buffer rotation, pivots
     DevStage* h_stage = nullptr;   // pinned copy read after the sort (stage statistics)
     MergeDesc* d_desc = nullptr;   // this rank's exchange+merge of the current stage, resolved on the GPU
@@ -260,7 +260,7 @@ int alloc_rank(msort_ctx* ctx, Rank& R, bool need_b1, bool need_stage) {
     CUDA_TRY(cudaMalloc(&R.d_desc, sizeof(MergeDesc)));
     CUDA_TRY(cudaMallocHost(&R.h_stage, sizeof(DevStage)));
     CUDA_TRY(cudaMallocHost(&R.h_pivot, 128 * sizeof(uint64_t)));
-    CUDA_TRY(cudaMallocHost(&R.h_trivial, 24 * sizeof(uint32_t)));
+    CUDA_TRY(cudaMallocHost(&R.h_trivial, kTrivialWords * sizeof(uint32_t)));
     CUDA_TRY(cudaMallocHost(&R.h_err, sizeof(int)));
     *R.h_err = 0;
     cudaEvent_t* evs[] = {&R.e_begin, &R.e_hist, &R.e_sorted, &R.e_end, &R.e_h2d0, &R.e_h2d1, &R.e_d2h0, &R.e_d2h1};
@@ -350,7 +350,7 @@ int radix_begin(msort_ctx* ctx, Rank& R, const void* src, uint64_t c) {
     CUDA_TRY(radix_prologue(src, c, ctx->kt, ws, R.st));
     ctx->tm.kernel_launches += 2;
     if (ctx->timing) CUDA_TRY(cudaEventRecord(R.e_hist, R.st));
-    if (ctx->skip_trivial) CUDA_TRY(cudaMemcpyAsync(R.h_trivial, ws.trivial, 24 * sizeof(uint32_t), cudaMemcpyDeviceToHost, R.st));
+    if (ctx->skip_trivial) CUDA_TRY(cudaMemcpyAsync(R.h_trivial, ws.trivial, kTrivialWords * sizeof(uint32_t), cudaMemcpyDeviceToHost, R.st));
     return MSORT_OK;
 }
 
@@ -416,7 +416,10 @@ int radix_passes(msort_ctx* ctx, Rank& R, const void* src, void* dst, void* tmp,
         const uint64_t maxbin = ctx->skip_trivial ? uint64_t(R.h_trivial[8 + pid]) : 0;
         const bool skewed = maxbin * 16 > c;
         const int mode = skew_mode();
-        const bool dominant = mode == 1 ? skewed : (mode == 0 || mode == 3 ? false : maxbin * 4 > c);
+        // (default: hot-4 when one digit holds > 1/4 of the keys or the 4 largest bins > 1/2 - e.g. the
+        // exponent byte of floats; a long tail of elevated digits, as in zipf, ranks faster by peer match)
+        const uint64_t top4 = ctx->skip_trivial ? uint64_t(R.h_trivial[24 + pid]) : 0;
+        const bool dominant = mode == 1 ? skewed : (mode == 0 || mode == 3 ? false : maxbin * 4 > c || top4 * 2 > c);
         bool atomic_rank = j == 0 || atomic_rank_ok(R.st);
         if (skewed && !dominant && mode != 3) atomic_rank = false;  // peer match
         const bool hot = dominant && atomic_rank;

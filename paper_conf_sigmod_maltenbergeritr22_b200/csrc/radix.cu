@@ -138,13 +138,14 @@ __global__ void __launch_bounds__(kRadix) scan_kernel(const uint32_t* __restrict
     if (uint64_t(v) == n) any_full = 1;
     // the 4 most frequent digit values (skewed passes rank them with one atomic
     // per warp row each), largest first
-    uint32_t top4 = 0, top_count = 0;
+    uint32_t top4 = 0, top_count = 0, top4_count = 0;
     bool taken = false;
     for (int q = 0; q < 4; ++q) {
         if (!taken) atomicMax(&max_bin, (static_cast<unsigned long long>(v) << 8) | unsigned(d));
         __syncthreads();
         const unsigned long long b = max_bin;
         if (q == 0) top_count = uint32_t(b >> 8);
+        top4_count += uint32_t(b >> 8);
         top4 |= uint32_t(b & 0xFF) << (8 * q);
         if (uint32_t(b & 0xFF) == uint32_t(d)) taken = true;
         __syncthreads();
@@ -155,6 +156,7 @@ __global__ void __launch_bounds__(kRadix) scan_kernel(const uint32_t* __restrict
         trivial[p] = any_full;
         trivial[8 + p] = top_count;  // size of the largest digit bin of the pass (skew)
         trivial[16 + p] = top4;      // the 4 most frequent digit values, one per byte
+        trivial[24 + p] = top4_count;  // keys on those 4 values
     }
 }
 
@@ -778,7 +780,7 @@ static uint32_t radix_group(int kt) { return key_bytes(kt) == 4 ? Cfg32::kGroup 
 
 static size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
-static size_t head_bytes() { return align_up(8 * 4 + 8 * 256 * 4 * 2 + 24 * 4, 256); }
+static size_t head_bytes() { return align_up(8 * 4 + 8 * 256 * 4 * 2 + kTrivialWords * 4, 256); }
 
 // Layout: head (counters, hist, bases, trivial) | group aggregates (zeroed per
 // sort) | status words (tagged, zeroed when the epoch wraps)
