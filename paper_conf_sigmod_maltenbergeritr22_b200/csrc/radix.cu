@@ -269,9 +269,12 @@ struct OsCfg {
 #define MSORT_LB_SLEEP_NS 32  // back-off of a look-back poll on an unpublished predecessor
 #endif
 #ifndef MSORT_BM32
-#define MSORT_BM32 0x7777777u  // peer-match ranking: items ranked by the ballot match (bit set; 3 of 4) vs smem atomicOr masks
+#define MSORT_BM32 0x7777777u  // peer-match ranking: items by the 8-ballot match (3 of 4); items in neither mask use smem atomicOr masks
 #endif
-#define MSORT_CFG32 OsCfg<MSORT_T32, MSORT_I32, MSORT_BM32, MSORT_B32, MSORT_W32, MSORT_G32, true>
+#ifndef MSORT_MM32
+#define MSORT_MM32 0x8888888u  // peer-match ranking: the 4th item of every 4 by __match_any_sync (ADU pipe)
+#endif
+#define MSORT_CFG32 OsCfg<MSORT_T32, MSORT_I32, (MSORT_BM32 | MSORT_MM32), MSORT_B32, MSORT_W32, MSORT_G32, true>
 #ifndef MSORT_CE64
 #define MSORT_CE64 true
 #endif
@@ -547,7 +550,10 @@ __global__ void __launch_bounds__(Cfg::kThreads, Cfg::kMinBlocks)
                 continue;
             }
             uint32_t peers;
-            if ((Cfg::kBallotMask >> i) & 1u) {
+            constexpr uint32_t kMatch = sizeof(U) == 4 ? MSORT_MM32 : 0u;  // items by match.any (ADU pipe)
+            if ((kMatch >> i) & 1u) {
+                peers = __match_any_sync(0xffffffffu, d);
+            } else if ((Cfg::kBallotMask >> i) & 1u) {
                 peers = ballot_match8(d);
             } else {
                 atomicOr(&s_match[warp][d], 1u << lane);
