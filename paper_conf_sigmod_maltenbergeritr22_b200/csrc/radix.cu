@@ -10,10 +10,10 @@
 //                    atomics of one warp instruction never collide on a bank
 //   scan_kernel      exclusive prefix per pass -> global digit bases (S2)
 //   onesweep_kernel  persistent blocks; per tile: block digit counts, stable
-//                    warp ranking (lane-ordered smem atomics, or atomicOr /
-//                    8-ballot peer masks), decoupled look-back across tiles
-//                    (32-bit group-relative status words, per-group bases)
-//                    for the global digit offset, smem staging, coalesced
+//                    warp ranking (lane-ordered smem atomics, or peer masks
+//                    from an 8-ballot match / match.any), decoupled look-back
+//                    across tiles (64-bit epoch-tagged status words, per-group
+//                    aggregates) for the global digit offset, smem staging, coalesced
 //                    scatter (S3); the next tile's keys load during the scatter
 // The float codec T (reading Q1) is applied on the first pass's load and T^-1
 // on the last pass's store (S1), so no separate codec pass touches HBM.
@@ -170,7 +170,8 @@ __global__ void __launch_bounds__(kRadix) scan_kernel(const uint32_t* __restrict
 // ~60 ADU cycles.  Per tile: per-warp digit counts first ("early counts"), the
 // tile aggregate is published before the ranking, and the ranking's atomic
 // returns the key's final smem slot (lane-ordered shared atomics, or a peer
-// match that mixes an 8-ballot match (ALU) with an smem atomicOr mask).
+// match that mixes an 8-ballot match (ALU) with match.any (ADU) and, for items
+// in neither mask, an smem atomicOr mask).
 //
 // Decoupled look-back: one 64-bit status word per (tile, digit),
 //   flag << 62 | tag << 32 | count       (tag = epoch << 4 | pass + 1)
